@@ -1,0 +1,279 @@
+"""Oracle-own TE-program builders (TEST INFRASTRUCTURE ONLY; see oracle/te.py header).
+
+The canonical programs follow SURVEY.md Appendix A (a restatement of the paper's models):
+  fig2()   PAPER.md Fig. 2 L628-633 (TE4 reads O3: the printed O4[i,rk] self-reference is a garble)
+  fig3()   PAPER.md Fig. 3 L970-982 (two GEMMs, horizontal transformation)
+  fig4()   PAPER.md Fig. 4 L1030-1050 (relu -> strided slice -> permute, vertical transformation)
+  bert()   BERT encoder (Table 2): 49 TEs per layer, post-LN, exact-erf GELU, eps 1e-12
+  mmoe()   MMoE (Table 2, ref [32]): 8 experts, 2 gates, 2 towers (sizes are a reading)
+  lstm()   stacked LSTM (Table 2, §8.4): torch.nn.LSTM semantics
+
+Placeholders are created immediately before their first use, so node ids are a deterministic
+function of the model; the product-side builder follows the same convention and the tests check
+that both produce the same node sequence.
+"""
+from __future__ import annotations
+
+
+class SpecBuilder:
+    def __init__(self):
+        self.nodes = []
+        self.outputs = []
+
+    def _add(self, n):
+        self.nodes.append(n)
+        return len(self.nodes) - 1
+
+    def ph(self, shape, dtype="f32", const=1):
+        return self._add(dict(op="placeholder", shape=list(shape), dtype=dtype, const=const))
+
+    def mm(self, a, b, trans_b=1, prec="f32"):
+        return self._add(dict(op="matmul", a=a, b=b, trans_b=trans_b, prec=prec))
+
+    def ew(self, fn, *ins, scalar=0.0):
+        return self._add({"op": "ew", "fn": fn, "in": list(ins), "scalar": float(scalar)})
+
+    def red(self, fn, x, axis, keepdim=1):
+        return self._add({"op": "reduce", "fn": fn, "in": x, "axis": axis, "keepdim": keepdim})
+
+    def reshape(self, x, shape):
+        return self._add({"op": "reshape", "in": x, "shape": list(shape)})
+
+    def permute(self, x, perm):
+        return self._add({"op": "permute", "in": x, "perm": list(perm)})
+
+    def slice(self, x, begin, end, stride):
+        return self._add({"op": "slice", "in": x, "begin": list(begin), "end": list(end), "stride": list(stride)})
+
+    def out(self, t):
+        self.outputs.append(t)
+
+    def spec(self):
+        return {"nodes": self.nodes, "outputs": list(self.outputs)}
+
+
+def fig2():
+    b = SpecBuilder()
+    I0 = b.ph((64, 64), const=0)
+    W0 = b.ph((64, 64))
+    O0 = b.mm(I0, W0, trans_b=0)          # TE0
+    O1 = b.ew("sigmoid", O0)              # TE1
+    W2 = b.ph((64, 64))
+    O2 = b.mm(O1, W2, trans_b=0)          # TE2
+    O3 = b.ew("add", O0, O2)              # TE3
+    W4 = b.ph((64, 256))
+    O4 = b.mm(O3, W4, trans_b=0)          # TE4
+    b.out(O4)
+    return b.spec(), dict(TE0=O0, TE1=O1, TE2=O2, TE3=O3, TE4=O4)
+
+
+def fig3():
+    b = SpecBuilder()
+    A1 = b.ph((4, 8), const=0)
+    B1 = b.ph((8, 16))
+    C1 = b.mm(A1, B1, trans_b=0)
+    A2 = b.ph((2, 8), const=0)
+    B2 = b.ph((8, 16))
+    C2 = b.mm(A2, B2, trans_b=0)
+    b.out(C1)
+    b.out(C2)
+    return b.spec(), dict(C1=C1, C2=C2, A1=A1, B1=B1, A2=A2, B2=B2)
+
+
+def fig4():
+    b = SpecBuilder()
+    A = b.ph((4, 8), const=0)
+    B = b.ew("relu", A)
+    C = b.slice(B, (0, 0), (4, 4), (2, 1))   # C[i,j] = B[2i, j], shape (2,4)
+    D = b.permute(C, (1, 0))                 # D[i,j] = C[j,i], shape (4,2)
+    b.out(D)
+    return b.spec(), dict(A=A, B=B, C=C, D=D)
+
+
+def _layernorm(b, x, H, eps, prefix_gamma, prefix_beta):
+    mu = b.red("mean", x, 1)
+    d = b.ew("sub", x, mu)
+    q = b.ew("mul", d, d)
+    v = b.red("mean", q, 1)
+    ve = b.ew("add_scalar", v, scalar=eps)
+    rs = b.ew("rsqrt", ve)
+    nrm = b.ew("mul", d, rs)
+    g = b.ph((H,))
+    gm = b.ew("mul", nrm, g)
+    be = b.ph((H,))
+    return b.ew("add", gm, be), (g, be)
+
+
+def bert_layer(b, X, cfg, params):
+    """Append one post-LN BERT encoder layer (49 TEs) to builder b.  params collects
+    placeholder ids by name."""
+    S, H, nh, F = cfg["seq"], cfg["hidden"], cfg["heads"], cfg["ffn"]
+    d = H // nh
+    prec = cfg["gemm_dtype"]
+    wd = cfg["gemm_dtype"]
+    qkv = []
+    for nm in ("q", "k", "v"):
+        W = b.ph((H, H), dtype=wd)
+        m0 = b.mm(X, W, 1, prec)
+        bb = b.ph((H,))
+        m1 = b.ew("add", m0, bb)
+        params["W" + nm], params["b" + nm] = W, bb
+        qkv.append(m1)
+    heads = []
+    for m1 in qkv:
+        r = b.reshape(m1, (S, nh, d))
+        heads.append(b.permute(r, (1, 0, 2)))
+    Qp, Kp, Vp = heads
+    Sc = b.mm(Qp, Kp, 1, prec)
+    Ss = b.ew("mul_scalar", Sc, scalar=1.0 / (d ** 0.5))
+    Mx = b.red("max", Ss, 2)
+    Sd = b.ew("sub", Ss, Mx)
+    E = b.ew("exp", Sd)
+    Z = b.red("sum", E, 2)
+    P = b.ew("div", E, Z)
+    Cx = b.mm(P, Vp, 0, prec)
+    Ct = b.permute(Cx, (1, 0, 2))
+    Cr = b.reshape(Ct, (S, H))
+    Wo = b.ph((H, H), dtype=wd)
+    A0 = b.mm(Cr, Wo, 1, prec)
+    bo = b.ph((H,))
+    A1 = b.ew("add", A0, bo)
+    R1 = b.ew("add", A1, X)
+    L1, (g1, be1) = _layernorm(b, R1, H, cfg["eps"], "g1", "be1")
+    W1 = b.ph((F, H), dtype=wd)
+    F0 = b.mm(L1, W1, 1, prec)
+    c1 = b.ph((F,))
+    F1 = b.ew("add", F0, c1)
+    F2 = b.ew("gelu_erf", F1)
+    W2 = b.ph((H, F), dtype=wd)
+    O0 = b.mm(F2, W2, 1, prec)
+    c2 = b.ph((H,))
+    O1 = b.ew("add", O0, c2)
+    R2 = b.ew("add", O1, L1)
+    Y, (g2, be2) = _layernorm(b, R2, H, cfg["eps"], "g2", "be2")
+    params.update(Wo=Wo, bo=bo, g1=g1, be1=be1, W1=W1, c1=c1, W2=W2, c2=c2, g2=g2, be2=be2)
+    return Y
+
+
+def bert(cfg, layers=None):
+    """BERT encoder over the post-embedding hidden state X [S, H].  Returns (spec, X id, list of
+    per-layer param-id dicts, output id)."""
+    b = SpecBuilder()
+    X = b.ph((cfg["seq"], cfg["hidden"]), const=0)
+    plist = []
+    h = X
+    for _ in range(layers if layers is not None else cfg["layers"]):
+        p = {}
+        h = bert_layer(b, h, cfg, p)
+        plist.append(p)
+    b.out(h)
+    return b.spec(), X, plist, h
+
+
+def bert_feed(X_id, plist, x, weights):
+    """Map placeholder ids -> stored arrays for bert()."""
+    feed = {X_id: x}
+    for p, w in zip(plist, weights):
+        for k, i in p.items():
+            feed[i] = w[k]
+    return feed
+
+
+def mmoe(cfg):
+    D, E, De, T, Th = cfg["d_in"], cfg["experts"], cfg["expert_dim"], cfg["tasks"], cfg["tower_hidden"]
+    B = cfg["batch"]
+    wd = cfg["w_dtype"]
+    b = SpecBuilder()
+    names = {}
+    x = b.ph((B, D), const=0)
+    names["x"] = x
+    ex = []
+    for e in range(E):
+        W = b.ph((De, D), dtype=wd)
+        m = b.mm(x, W, 1, "f32")
+        bb = b.ph((De,))
+        a = b.ew("add", m, bb)
+        ex.append(b.ew("relu", a))
+        names[f"We{e}"], names[f"be{e}"] = W, bb
+    gates = []
+    for k in range(T):
+        W = b.ph((E, D), dtype=wd)
+        m = b.mm(x, W, 1, "f32")
+        bb = b.ph((E,))
+        a = b.ew("add", m, bb)
+        mx = b.red("max", a, 1)
+        sd = b.ew("sub", a, mx)
+        ee = b.ew("exp", sd)
+        z = b.red("sum", ee, 1)
+        gates.append(b.ew("div", ee, z))
+        names[f"Wg{k}"], names[f"bg{k}"] = W, bb
+    outs = []
+    for k in range(T):
+        acc = None
+        for e in range(E):
+            s = b.slice(gates[k], (0, e), (B, e + 1), (1, 1))
+            p = b.ew("mul", s, ex[e])
+            acc = p if acc is None else b.ew("add", acc, p)
+        Wt = b.ph((Th, De), dtype=wd)
+        t0 = b.mm(acc, Wt, 1, "f32")
+        bt = b.ph((Th,))
+        t1 = b.ew("add", t0, bt)
+        t2 = b.ew("relu", t1)
+        Wo = b.ph((1, Th), dtype=wd)
+        y0 = b.mm(t2, Wo, 1, "f32")
+        bo = b.ph((1,))
+        y1 = b.ew("add", y0, bo)
+        b.out(y1)
+        outs.append(y1)
+        names[f"Wt{k}"], names[f"bt{k}"], names[f"Wo{k}"], names[f"bo{k}"] = Wt, bt, Wo, bo
+    return b.spec(), names, outs
+
+
+def lstm(cfg):
+    """Stacked LSTM, torch.nn.LSTM gate order i, f, g, o; h0 = c0 = 0 supplied as placeholders.
+    Per cell-step: 2 GEMVs + 3 adds + 4 slices + 4 activations + 5 state ops."""
+    T, H, I, L = cfg["steps"], cfg["hidden"], cfg["input"], cfg["layers"]
+    wd = cfg["w_dtype"]
+    b = SpecBuilder()
+    names = {}
+    X = b.ph((T, I), const=0)
+    names["X"] = X
+    W, U, bi, bh, h, c = [], [], [], [], [], []
+    for n in range(L):
+        W.append(b.ph((4 * H, I if n == 0 else H), dtype=wd))
+        U.append(b.ph((4 * H, H), dtype=wd))
+        bi.append(b.ph((4 * H,)))
+        bh.append(b.ph((4 * H,)))
+        h.append(b.ph((1, H), const=0))
+        c.append(b.ph((1, H), const=0))
+        names.update({f"W{n}": W[n], f"U{n}": U[n], f"bih{n}": bi[n], f"bhh{n}": bh[n], f"h0_{n}": h[n],
+                      f"c0_{n}": c[n]})
+    top = []
+    for t in range(T):
+        x = b.slice(X, (t, 0), (t + 1, I), (1, 1))
+        for n in range(L):
+            g0 = b.mm(x, W[n], 1, "f32")
+            g1 = b.ew("add", g0, bi[n])
+            g2 = b.mm(h[n], U[n], 1, "f32")
+            g3 = b.ew("add", g1, g2)
+            g4 = b.ew("add", g3, bh[n])
+            gi = b.slice(g4, (0, 0), (1, H), (1, 1))
+            gf = b.slice(g4, (0, H), (1, 2 * H), (1, 1))
+            gg = b.slice(g4, (0, 2 * H), (1, 3 * H), (1, 1))
+            go = b.slice(g4, (0, 3 * H), (1, 4 * H), (1, 1))
+            i_ = b.ew("sigmoid", gi)
+            f_ = b.ew("sigmoid", gf)
+            g_ = b.ew("tanh", gg)
+            o_ = b.ew("sigmoid", go)
+            fc = b.ew("mul", f_, c[n])
+            ig = b.ew("mul", i_, g_)
+            c[n] = b.ew("add", fc, ig)
+            tc = b.ew("tanh", c[n])
+            h[n] = b.ew("mul", o_, tc)
+            x = h[n]
+        top.append(x)
+        b.out(x)
+    for n in range(L):
+        b.out(h[n])
+        b.out(c[n])
+    return b.spec(), names, top, list(h), list(c)

@@ -1,0 +1,229 @@
+"""Seeded synthetic inputs shared by the oracle tests, the GPU parity tests and bench.py.
+
+This module holds NO arithmetic of the method (no TE semantics, no analysis, no partitioning).
+It only draws random numbers from documented seeds and rounds them ONCE to their storage dtype,
+so that both sides of every parity check consume bit-identical stored values
+(SURVEY.md §8(c) item 9, §8(d) "Synthetic inputs").
+
+Generator: numpy.random.Generator(PCG64(seed)) in fp64, then fp64 -> fp32 (numpy RNE) and, for bf16
+storage, fp32 -> bf16 by round-to-nearest-even on the bit pattern.  Seeds: inputs = 1234,
+weights = 1000 * layer + slot (slot numbers below).
+
+Workload recipes:
+  * BERT (Table 2, §7.1): X ~ N(0,1) fp32 is the post-embedding hidden
+    state; GEMM weights W ~ N(0, 1/K) stored [N, K]; biases N(0, 0.02^2); LN gamma = 1 + N(0, 0.1^2),
+    beta = N(0, 0.1^2).
+  * LSTM (Table 2): x ~ N(0,1) [T, 256]; W_ih, W_hh, b_ih, b_hh ~ U(+-1/sqrt(H)) (PyTorch
+    default init, contractive; SURVEY §8(c) tolerances).
+  * MMoE (Table 2, reading in DESIGN.md): x ~ N(0,1) [1, 100]; every weight ~ N(0, 1/K),
+    biases N(0, 0.02^2).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+INPUT_SEED = 1234
+
+# ---------------------------------------------------------------- configs (BASELINE.json configs)
+BERT_TINY = dict(name="bert_tiny", seq=32, hidden=64, heads=2, ffn=256, layers=1, gemm_dtype="f32",
+                 eps=1e-12)
+BERT_BASE = dict(name="bert_base", seq=128, hidden=768, heads=12, ffn=3072, layers=12, gemm_dtype="bf16",
+                 eps=1e-12)
+LSTM_CFG = dict(name="lstm", steps=100, hidden=256, input=256, layers=10, w_dtype="bf16")
+MMOE_CFG = dict(name="mmoe", d_in=100, experts=8, expert_dim=16, tasks=2, tower_hidden=8, batch=1,
+                w_dtype="f32")
+
+# weight slot numbers inside one BERT layer (seed = 1000*layer + slot)
+BERT_SLOTS = dict(Wq=1, bq=2, Wk=3, bk=4, Wv=5, bv=6, Wo=7, bo=8, g1=9, be1=10, W1=11, c1=12, W2=13, c2=14,
+                  g2=15, be2=16)
+
+
+def rng(seed: int) -> np.random.Generator:
+    return np.random.Generator(np.random.PCG64(seed))
+
+
+# ---------------------------------------------------------------- storage rounding (bit level)
+def f32_to_bf16_bits(x) -> np.ndarray:
+    """fp32 -> bf16 bit pattern (uint16), round-to-nearest-even on the bits (finite inputs)."""
+    u = np.ascontiguousarray(np.asarray(x, dtype=np.float32)).view(np.uint32).astype(np.uint64)
+    u = (u + 0x7FFF + ((u >> 16) & 1)) >> 16
+    return u.astype(np.uint16)
+
+
+def bf16_bits_to_f32(b) -> np.ndarray:
+    b = np.asarray(b, dtype=np.uint16).astype(np.uint32) << 16
+    return b.view(np.float32)
+
+
+def to_storage(x, dtype: str) -> np.ndarray:
+    """Round fp64 draws once to the storage dtype; returns float32 values exactly representable
+    in `dtype` ('f32' or 'bf16')."""
+    x32 = np.asarray(x, dtype=np.float64).astype(np.float32)
+    if dtype == "f32":
+        return x32
+    if dtype == "bf16":
+        return bf16_bits_to_f32(f32_to_bf16_bits(x32))
+    raise ValueError(dtype)
+
+
+def normal(seed, shape, std=1.0, mean=0.0, dtype="f32"):
+    return to_storage(mean + std * rng(seed).standard_normal(shape), dtype)
+
+
+def uniform(seed, shape, bound, dtype="f32"):
+    return to_storage(rng(seed).uniform(-bound, bound, size=shape), dtype)
+
+
+def small_ints(seed, shape, lo=-2, hi=2, dtype="f32"):
+    """Integer-valued draws in [lo, hi]: exact in bf16 and fp32, so GEMMs over them are exact."""
+    return to_storage(rng(seed).integers(lo, hi + 1, size=shape).astype(np.float64), dtype)
+
+
+# ---------------------------------------------------------------- BERT
+def bert_layer_weights(cfg: dict, layer: int, integer: bool = False) -> dict:
+    H, F = cfg["hidden"], cfg["ffn"]
+    wd = cfg["gemm_dtype"]
+    s = lambda k: 1000 * layer + BERT_SLOTS[k]
+    if integer:
+        w = lambda k, shp: small_ints(s(k), shp, dtype=wd)
+        v = lambda k, shp: small_ints(s(k), shp, dtype="f32")
+        g = lambda k, shp: small_ints(s(k), shp, 0, 2, dtype="f32")
+    else:
+        w = lambda k, shp: normal(s(k), shp, std=1.0 / np.sqrt(shp[1]), dtype=wd)
+        v = lambda k, shp: normal(s(k), shp, std=0.02)
+        g = lambda k, shp: normal(s(k), shp, std=0.1, mean=1.0)
+    p = dict(Wq=w("Wq", (H, H)), bq=v("bq", (H,)), Wk=w("Wk", (H, H)), bk=v("bk", (H,)),
+             Wv=w("Wv", (H, H)), bv=v("bv", (H,)), Wo=w("Wo", (H, H)), bo=v("bo", (H,)),
+             g1=g("g1", (H,)), W1=w("W1", (F, H)), c1=v("c1", (F,)), W2=w("W2", (H, F)), c2=v("c2", (H,)),
+             g2=g("g2", (H,)))
+    if integer:
+        p["be1"] = small_ints(s("be1"), (H,))
+        p["be2"] = small_ints(s("be2"), (H,))
+    else:
+        p["be1"] = normal(s("be1"), (H,), std=0.1)
+        p["be2"] = normal(s("be2"), (H,), std=0.1)
+    return p
+
+
+def bert_input(cfg: dict, seed: int = INPUT_SEED, batch: int = 1) -> np.ndarray:
+    shape = (cfg["seq"], cfg["hidden"]) if batch == 1 else (batch, cfg["seq"], cfg["hidden"])
+    return normal(seed, shape)
+
+
+def bert_weights(cfg: dict, integer: bool = False) -> list:
+    return [bert_layer_weights(cfg, l, integer) for l in range(cfg["layers"])]
+
+
+# ---------------------------------------------------------------- LSTM
+def lstm_params(cfg: dict, w_dtype: str | None = None) -> list:
+    H, I = cfg["hidden"], cfg["input"]
+    wd = w_dtype or cfg["w_dtype"]
+    b = 1.0 / np.sqrt(H)
+    out = []
+    for n in range(cfg["layers"]):
+        out.append(dict(W=uniform(1000 * n + 1, (4 * H, I if n == 0 else H), b, wd),
+                        U=uniform(1000 * n + 2, (4 * H, H), b, wd),
+                        b_ih=uniform(1000 * n + 3, (4 * H,), b),
+                        b_hh=uniform(1000 * n + 4, (4 * H,), b)))
+    return out
+
+
+def lstm_input(cfg: dict, seed: int = INPUT_SEED) -> np.ndarray:
+    return normal(seed, (cfg["steps"], cfg["input"]))
+
+
+# ---------------------------------------------------------------- MMoE
+def mmoe_params(cfg: dict) -> dict:
+    D, E, De, T, Th = cfg["d_in"], cfg["experts"], cfg["expert_dim"], cfg["tasks"], cfg["tower_hidden"]
+    wd = cfg["w_dtype"]
+    p = {}
+    for e in range(E):
+        p[f"We{e}"] = normal(100 + e, (De, D), std=1 / np.sqrt(D), dtype=wd)
+        p[f"be{e}"] = normal(200 + e, (De,), std=0.02)
+    for k in range(T):
+        p[f"Wg{k}"] = normal(300 + k, (E, D), std=1 / np.sqrt(D), dtype=wd)
+        p[f"bg{k}"] = normal(400 + k, (E,), std=0.02)
+        p[f"Wt{k}"] = normal(500 + k, (Th, De), std=1 / np.sqrt(De), dtype=wd)
+        p[f"bt{k}"] = normal(600 + k, (Th,), std=0.02)
+        p[f"Wo{k}"] = normal(700 + k, (1, Th), std=1 / np.sqrt(Th), dtype=wd)
+        p[f"bo{k}"] = normal(800 + k, (1,), std=0.02)
+    return p
+
+
+def mmoe_input(cfg: dict, seed: int = INPUT_SEED) -> np.ndarray:
+    return normal(seed, (cfg["batch"], cfg["d_in"]))
+
+
+# ---------------------------------------------------------------- random TE-program specs
+# Spec format (a plain data format consumed by oracle/te.py and by the binding's spec builder):
+#   {"nodes": [node, ...], "outputs": [ids]}, node ids = list positions (creation order = topological)
+#   placeholder: {"op":"placeholder","shape":[..],"dtype":"f32"|"bf16","const":0|1}
+#   matmul:      {"op":"matmul","a":i,"b":j,"trans_b":0|1,"prec":"f32"|"bf16"}
+#   ew:          {"op":"ew","fn":name,"in":[ids],"scalar":x}
+#   reduce:      {"op":"reduce","fn":"sum"|"max"|"mean","in":i,"axis":k,"keepdim":0|1}
+#   reshape:     {"op":"reshape","in":i,"shape":[..]}
+#   permute:     {"op":"permute","in":i,"perm":[..]}
+#   slice:       {"op":"slice","in":i,"begin":[..],"end":[..],"stride":[..]}
+UNARY = ["exp", "tanh", "sigmoid", "relu", "gelu_erf", "rsqrt", "neg"]
+BINARY = ["add", "sub", "mul", "div", "max"]
+SCALAR = ["add_scalar", "mul_scalar"]
+
+
+def random_spec(seed: int, n_ops: int = 12, dim_choices=(2, 3, 4, 5)) -> dict:
+    """Random 2-D TE program over small shapes (structure only; shapes kept consistent here so the
+    builder never has to reject).  Used for analysis property tests and generic-executor parity."""
+    r = rng(seed)
+    nodes, shapes = [], []
+
+    def add(node, shape):
+        nodes.append(node)
+        shapes.append(tuple(shape))
+        return len(nodes) - 1
+
+    M, K = int(r.choice(dim_choices)), int(r.choice(dim_choices))
+    x = add(dict(op="placeholder", shape=[M, K], dtype="f32", const=0), (M, K))
+    live = [x]
+    for _ in range(n_ops):
+        kind = r.choice(["mm", "un", "bin", "red", "perm", "scal"])
+        src = int(r.choice(live))
+        shp = shapes[src]
+        if len(shp) != 2:
+            continue
+        if kind == "mm":
+            N = int(r.choice(dim_choices))
+            w = add(dict(op="placeholder", shape=[N, shp[1]], dtype="f32", const=1), (N, shp[1]))
+            nid = add(dict(op="matmul", a=src, b=w, trans_b=1, prec="f32"), (shp[0], N))
+        elif kind == "un":
+            fn = str(r.choice(["tanh", "sigmoid", "relu", "neg", "exp"]))
+            nid = add(dict(op="ew", fn=fn, **{"in": [src]}, scalar=0.0), shp)
+        elif kind == "scal":
+            fn = str(r.choice(SCALAR))
+            nid = add(dict(op="ew", fn=fn, **{"in": [src]}, scalar=float(r.choice([0.5, -1.0, 2.0]))), shp)
+        elif kind == "bin":
+            same = [i for i in live if shapes[i] == shp and i != src]
+            if same:
+                other = int(r.choice(same))
+            else:
+                other = add(dict(op="placeholder", shape=[shp[1]], dtype="f32", const=1), (shp[1],))
+            fn = str(r.choice(["add", "sub", "mul", "max"]))
+            nid = add(dict(op="ew", fn=fn, **{"in": [src, other]}, scalar=0.0), shp)
+        elif kind == "red":
+            fn = str(r.choice(["sum", "max", "mean"]))
+            nid = add(dict(op="reduce", fn=fn, **{"in": src}, axis=1, keepdim=1), (shp[0], 1))
+        else:
+            nid = add(dict(op="permute", **{"in": src}, perm=[1, 0]), (shp[1], shp[0]))
+        live.append(nid)
+    return {"nodes": nodes, "outputs": [len(nodes) - 1]}
+
+
+def spec_inputs(spec: dict, seed: int, integer: bool = False) -> dict:
+    """Seeded values for every placeholder of a spec (dict id -> float32 array in storage dtype)."""
+    out = {}
+    for i, n in enumerate(spec["nodes"]):
+        if n["op"] != "placeholder":
+            continue
+        if integer:
+            out[i] = small_ints(seed * 7919 + i, tuple(n["shape"]), dtype=n["dtype"])
+        else:
+            out[i] = normal(seed * 7919 + i, tuple(n["shape"]), std=0.5, dtype=n["dtype"])
+    return out
