@@ -1,0 +1,205 @@
+"""TE-program builders for the evaluated models, through the C ABI (argument marshalling only).
+
+Each builder creates placeholders immediately before their first use -- the same convention as
+SURVEY.md Appendix A -- so node ids are a deterministic function of the model.
+  bert      BERT encoder, 49 TEs per layer (Table 2; post-LN, erf GELU, eps 1e-12)
+  mmoe      multi-gate mixture of experts (Table 2)
+  lstm      stacked LSTM, torch.nn.LSTM gate order (Table 2, §8.4)
+  fig2      PAPER.md Fig. 2 (L628-633)
+  from_spec a plain-data TE program (synth.random_spec format)
+"""
+from __future__ import annotations
+
+from . import _lib as L
+
+_DT = {"f32": L.F32, "bf16": L.BF16}
+
+
+def _layernorm(g, x, H, eps, names, gk, bk):
+    mu = g.reduce("mean", x, 1)
+    d = g.ew("sub", x, mu)
+    q = g.ew("mul", d, d)
+    v = g.reduce("mean", q, 1)
+    ve = g.ew("add_scalar", v, scalar=eps)
+    rs = g.ew("rsqrt", ve)
+    n = g.ew("mul", d, rs)
+    gm = g.placeholder((H,))
+    a = g.ew("mul", n, gm)
+    be = g.placeholder((H,))
+    names[gk], names[bk] = gm, be
+    return g.ew("add", a, be)
+
+
+def bert_layer(g, X, cfg, names):
+    S, H, nh, F = cfg["seq"], cfg["hidden"], cfg["heads"], cfg["ffn"]
+    d = H // nh
+    prec = _DT[cfg["gemm_dtype"]]
+    qkv = []
+    for nm in ("q", "k", "v"):
+        W = g.placeholder((H, H), prec)
+        m = g.matmul(X, W, True, prec)
+        b = g.placeholder((H,))
+        qkv.append(g.ew("add", m, b))
+        names["W" + nm], names["b" + nm] = W, b
+    Qp, Kp, Vp = [g.permute(g.reshape(t, (S, nh, d)), (1, 0, 2)) for t in qkv]
+    Sc = g.matmul(Qp, Kp, True, prec)
+    Ss = g.ew("mul_scalar", Sc, scalar=1.0 / (d ** 0.5))
+    Mx = g.reduce("max", Ss, 2)
+    Sd = g.ew("sub", Ss, Mx)
+    E = g.ew("exp", Sd)
+    Z = g.reduce("sum", E, 2)
+    P = g.ew("div", E, Z)
+    Cx = g.matmul(P, Vp, False, prec)
+    Cr = g.reshape(g.permute(Cx, (1, 0, 2)), (S, H))
+    Wo = g.placeholder((H, H), prec)
+    A0 = g.matmul(Cr, Wo, True, prec)
+    bo = g.placeholder((H,))
+    R1 = g.ew("add", g.ew("add", A0, bo), X)
+    L1 = _layernorm(g, R1, H, cfg["eps"], names, "g1", "be1")
+    W1 = g.placeholder((F, H), prec)
+    F0 = g.matmul(L1, W1, True, prec)
+    c1 = g.placeholder((F,))
+    F2 = g.ew("gelu_erf", g.ew("add", F0, c1))
+    W2 = g.placeholder((H, F), prec)
+    O0 = g.matmul(F2, W2, True, prec)
+    c2 = g.placeholder((H,))
+    R2 = g.ew("add", g.ew("add", O0, c2), L1)
+    names.update(Wo=Wo, bo=bo, W1=W1, c1=c1, W2=W2, c2=c2)
+    return _layernorm(g, R2, H, cfg["eps"], names, "g2", "be2")
+
+
+def bert(cfg, layers=None):
+    """Returns (graph, X id, [per-layer name->id], output id)."""
+    g = L.Graph()
+    X = g.placeholder((cfg["seq"], cfg["hidden"]), L.F32, const=False)
+    plist = []
+    h = X
+    for _ in range(cfg["layers"] if layers is None else layers):
+        names = {}
+        h = bert_layer(g, h, cfg, names)
+        plist.append(names)
+    g.mark_output(h)
+    return g, X, plist, h
+
+
+def mmoe(cfg):
+    D, E, De, T, Th, B = (cfg[k] for k in ("d_in", "experts", "expert_dim", "tasks", "tower_hidden", "batch"))
+    wd = _DT[cfg["w_dtype"]]
+    g = L.Graph()
+    names = {}
+    x = g.placeholder((B, D), L.F32, const=False)
+    names["x"] = x
+    ex = []
+    for e in range(E):
+        W = g.placeholder((De, D), wd)
+        m = g.matmul(x, W, True, L.F32)
+        b = g.placeholder((De,))
+        ex.append(g.ew("relu", g.ew("add", m, b)))
+        names[f"We{e}"], names[f"be{e}"] = W, b
+    gates = []
+    for k in range(T):
+        W = g.placeholder((E, D), wd)
+        m = g.matmul(x, W, True, L.F32)
+        b = g.placeholder((E,))
+        a = g.ew("add", m, b)
+        mx = g.reduce("max", a, 1)
+        ee = g.ew("exp", g.ew("sub", a, mx))
+        z = g.reduce("sum", ee, 1)
+        gates.append(g.ew("div", ee, z))
+        names[f"Wg{k}"], names[f"bg{k}"] = W, b
+    outs = []
+    for k in range(T):
+        acc = None
+        for e in range(E):
+            s = g.slice(gates[k], (0, e), (B, e + 1), (1, 1))
+            p = g.ew("mul", s, ex[e])
+            acc = p if acc is None else g.ew("add", acc, p)
+        Wt = g.placeholder((Th, De), wd)
+        t0 = g.matmul(acc, Wt, True, L.F32)
+        bt = g.placeholder((Th,))
+        t2 = g.ew("relu", g.ew("add", t0, bt))
+        Wo = g.placeholder((1, Th), wd)
+        y0 = g.matmul(t2, Wo, True, L.F32)
+        bo = g.placeholder((1,))
+        y = g.ew("add", y0, bo)
+        g.mark_output(y)
+        outs.append(y)
+        names[f"Wt{k}"], names[f"bt{k}"], names[f"Wo{k}"], names[f"bo{k}"] = Wt, bt, Wo, bo
+    return g, names, outs
+
+
+def lstm(cfg):
+    T, H, I, Ln = cfg["steps"], cfg["hidden"], cfg["input"], cfg["layers"]
+    wd = _DT[cfg["w_dtype"]]
+    g = L.Graph()
+    names = {}
+    X = g.placeholder((T, I), L.F32, const=False)
+    names["X"] = X
+    W, U, bi, bh, h, c = [], [], [], [], [], []
+    for n in range(Ln):
+        W.append(g.placeholder((4 * H, I if n == 0 else H), wd))
+        U.append(g.placeholder((4 * H, H), wd))
+        bi.append(g.placeholder((4 * H,)))
+        bh.append(g.placeholder((4 * H,)))
+        h.append(g.placeholder((1, H), L.F32, const=False))
+        c.append(g.placeholder((1, H), L.F32, const=False))
+        names.update({f"W{n}": W[n], f"U{n}": U[n], f"bih{n}": bi[n], f"bhh{n}": bh[n], f"h0_{n}": h[n],
+                      f"c0_{n}": c[n]})
+    top = []
+    for t in range(T):
+        x = g.slice(X, (t, 0), (t + 1, I), (1, 1))
+        for n in range(Ln):
+            g1 = g.ew("add", g.matmul(x, W[n], True, L.F32), bi[n])
+            g4 = g.ew("add", g.ew("add", g1, g.matmul(h[n], U[n], True, L.F32)), bh[n])
+            gi, gf, gg, go = (g.slice(g4, (0, k * H), (1, (k + 1) * H), (1, 1)) for k in range(4))
+            i_, f_, g_, o_ = g.ew("sigmoid", gi), g.ew("sigmoid", gf), g.ew("tanh", gg), g.ew("sigmoid", go)
+            c[n] = g.ew("add", g.ew("mul", f_, c[n]), g.ew("mul", i_, g_))
+            h[n] = g.ew("mul", o_, g.ew("tanh", c[n]))
+            x = h[n]
+        top.append(x)
+        g.mark_output(x)
+    for n in range(Ln):
+        g.mark_output(h[n])
+        g.mark_output(c[n])
+    return g, names, top, list(h), list(c)
+
+
+def fig2():
+    g = L.Graph()
+    I0 = g.placeholder((64, 64), L.F32, const=False)
+    W0 = g.placeholder((64, 64))
+    O0 = g.matmul(I0, W0, False)
+    O1 = g.ew("sigmoid", O0)
+    W2 = g.placeholder((64, 64))
+    O2 = g.matmul(O1, W2, False)
+    O3 = g.ew("add", O0, O2)
+    W4 = g.placeholder((64, 256))
+    O4 = g.matmul(O3, W4, False)
+    g.mark_output(O4)
+    return g, dict(TE0=O0, TE1=O1, TE2=O2, TE3=O3, TE4=O4)
+
+
+def from_spec(spec):
+    """Build a graph from the plain-data spec format documented in synth/__init__.py."""
+    g = L.Graph()
+    for n in spec["nodes"]:
+        op = n["op"]
+        if op == "placeholder":
+            g.placeholder(n["shape"], _DT[n["dtype"]], bool(n["const"]))
+        elif op == "matmul":
+            g.matmul(n["a"], n["b"], bool(n["trans_b"]), _DT[n["prec"]])
+        elif op == "ew":
+            g.ew(n["fn"], *n["in"], scalar=n.get("scalar", 0.0))
+        elif op == "reduce":
+            g.reduce(n["fn"], n["in"], n["axis"], bool(n["keepdim"]))
+        elif op == "reshape":
+            g.reshape(n["in"], n["shape"])
+        elif op == "permute":
+            g.permute(n["in"], n["perm"])
+        elif op == "slice":
+            g.slice(n["in"], n["begin"], n["end"], n["stride"])
+        else:
+            raise ValueError(op)
+    for o in spec["outputs"]:
+        g.mark_output(o)
+    return g

@@ -1,0 +1,174 @@
+"""CPU tests: libsouffle loads, exports every symbol of include/souffle.h, and its analysis /
+partition / index maps / horizontal groups are bit-exact with the oracle (no GPU needed)."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import analysis as an
+from oracle import graphs as og
+from oracle import te
+from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_header_symbol(lib):
+    hdr = open(os.path.join(ROOT, "include", "souffle.h")).read()
+    declared = sorted(set(re.findall(r"\b(souffle_[a-z0-9_]+)\s*\(", hdr)))
+    assert len(declared) >= 30
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert sorted(declared) == L.EXPORTS
+    assert b"sm_100a" in lib.souffle_version()
+
+
+def test_error_paths(lib):
+    g = L.Graph()
+    a = g.placeholder((4, 8))
+    b = g.placeholder((5, 8))
+    with pytest.raises(L.SouffleError) as e:
+        g.matmul(a, b, trans_b=False)
+    assert e.value.code == 2
+    with pytest.raises(L.SouffleError):
+        g.ew("add", a, 99)
+    with pytest.raises(L.SouffleError) as e:
+        g.partition()                      # no outputs
+    assert e.value.code == 6
+    c = g.matmul(a, b, trans_b=True)
+    g.mark_output(c)
+    p = g.partition()
+    assert p.workspace_bytes() > 0
+    with pytest.raises(L.SouffleError) as e:
+        p.run(0x1000)                      # not initialised
+    assert e.value.code in (1, 6)
+
+
+def _oracle_dev(d):
+    return dict(rule=d.rule, capacity_C=d.capacity_C, num_sms=d.num_sms, smem_per_sm=d.smem_per_sm,
+                smem_reserved_per_block=d.smem_reserved_per_block, regs_per_sm=d.regs_per_sm,
+                max_threads_per_sm=d.max_threads_per_sm, max_blocks_per_sm=d.max_blocks_per_sm)
+
+
+def _check_plan_vs_oracle(spec, plan, dev, check_maps=True):
+    info = an.classify(spec)
+    n = len(spec["nodes"])
+    assert plan.num_nodes() == n
+    res = {}
+    for i in range(n):
+        ti = plan.te_info(i)
+        assert ti["dep"] == info[i]["dep"], i
+        assert ti["ci"] == info[i]["ci"], i
+        assert ti["ops"] == info[i]["ops"], i
+        assert ti["accesses"] == info[i]["accesses"], i
+        res[i] = (ti["grid"], ti["smem"], ti["regs"], ti["threads"])
+    order = an.bfs_order(spec)
+    assert plan.bfs_order() == order
+    assign = an.partition(spec, res, _oracle_dev(dev), order=order, info=info)
+    assert plan.assignment() == assign
+    assert plan.num_subprograms() == (max(assign) + 1 if order else 0)
+    reuse = an.reuse_sets(spec)
+    for t in range(n):
+        cs, kind = plan.reuse_set(t)
+        if t in reuse:
+            assert (cs, kind) == reuse[t], t
+        else:
+            assert kind == -1
+    lv = an.levels(spec)
+    gid, kinds = an.hgroups(spec, assign)
+    for t in range(n):
+        l, g, k = plan.hgroup(t)
+        assert l == lv[t] and g == gid[t] and (k == (kinds[g] if g >= 0 else -1)), t
+    if check_maps:
+        shapes = te.infer_shapes(spec)
+        for t, nd in enumerate(spec["nodes"]):
+            if nd["op"] in an.OR_OPS:
+                for s in an.te_inputs(nd):
+                    ref = an.index_map(spec, t, s)
+                    got = plan.index_map(t, s, int(np.prod(shapes[t])))
+                    assert got == ref, (t, s)
+
+
+def test_fig2_paper_rule_partition():
+    spec, ids = og.fig2()
+    g, pids = M.fig2()
+    for name in ("TE0", "TE2", "TE4"):
+        grid = 64 if name == "TE4" else 16
+        g.set_te_resources(pids[name], grid, 1024, 0, 0)
+    dev = L.paper_device(48 * 1024)
+    plan = g.partition(dev)
+    a = plan.assignment()
+    assert [a[pids[k]] for k in ("TE0", "TE1", "TE2", "TE3", "TE4")] == [0, 0, 0, 0, 1]
+    _check_plan_vs_oracle(spec, plan, dev)
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_random_programs_bit_exact(seed):
+    spec = synth.random_spec(seed, n_ops=30)
+    g = M.from_spec(spec)
+    dev = L.device_b200()
+    plan = g.partition(dev)
+    _check_plan_vs_oracle(spec, plan, dev)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_random_programs_paper_rule_with_overrides(seed):
+    """Random resource vectors including exact equality at the capacity boundary."""
+    spec = synth.random_spec(100 + seed, n_ops=30)
+    g = M.from_spec(spec)
+    r = synth.rng(seed)
+    info = an.classify(spec)
+    C = 48 * 1024
+    for i, nd in enumerate(spec["nodes"]):
+        if nd["op"] != "placeholder" and info[i]["ci"]:
+            grid = int(r.choice([8, 16, 24, 48, 49, 64]))
+            g.set_te_resources(i, grid, 1024, 32, 128)
+    dev = L.paper_device(C)
+    plan = g.partition(dev)
+    _check_plan_vs_oracle(spec, plan, dev)
+
+
+@pytest.mark.parametrize("cfg", [synth.BERT_TINY, dict(synth.BERT_BASE, layers=2)])
+def test_bert_graph_matches_oracle_builder_and_analysis(cfg):
+    spec, X, plist, y = og.bert(cfg, layers=cfg["layers"])
+    g, gX, gplist, gy = M.bert(cfg)
+    assert g.num_nodes() == len(spec["nodes"]) and gX == X and gy == y and gplist == plist
+    shapes = te.infer_shapes(spec)
+    opmap = {"placeholder": 0, "matmul": 1, "ew": 2, "reduce": 3, "reshape": 4, "permute": 5, "slice": 6}
+    for i, nd in enumerate(spec["nodes"]):
+        op, shp, dt = g.node(i)
+        assert op == opmap[nd["op"]] and shp == shapes[i], i
+    dev = L.device_b200()
+    plan = g.partition(dev)
+    _check_plan_vs_oracle(spec, plan, dev, check_maps=cfg["layers"] == 1)
+
+
+def test_mmoe_and_lstm_graphs_one_subprogram():
+    for build_o, build_p, cfg in ((og.mmoe, M.mmoe, synth.MMOE_CFG),
+                                  (og.lstm, M.lstm, dict(synth.LSTM_CFG, steps=4))):
+        spec = build_o(cfg)[0]
+        g = build_p(cfg)[0]
+        assert g.num_nodes() == len(spec["nodes"])
+        dev = L.device_b200()
+        plan = g.partition(dev)
+        assert plan.num_subprograms() == 1            # Table 5: one kernel
+        _check_plan_vs_oracle(spec, plan, dev, check_maps=False)
+
+
+def test_bert_base_lowering_structure():
+    g, X, plist, y = M.bert(synth.BERT_BASE)
+    plan = g.partition(L.device_b200())
+    txt = plan.describe()
+    info = plan.exec_info()
+    assert plan.num_subprograms() == 1
+    assert info["launches"] == 1                     # whole model = one persistent kernel
+    assert txt.count("ATTN") == 12
+    assert txt.count("GEMM_TC") == 48                 # QKV (horizontal), out-proj, FFN1, FFN2 per layer
+    assert "mm " in txt and "tmaA" in txt
+    v0 = g.partition(L.device_b200(), flags=L.FLAG_UNFUSED).exec_info()
+    te_count = plan.num_tes()
+    assert v0["launches"] == te_count                 # V0: one kernel per TE (Fig. 5(a))

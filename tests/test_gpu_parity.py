@@ -1,0 +1,145 @@
+"""GPU parity: the fused sm_100a path (through the C ABI) against the CPU fp64 oracle on the same
+seeded inputs.  Tolerances (BASELINE.json north_star):
+  * integer / GEMM-only stages with inputs in {-2..2}: bit-exact
+  * fp32 paths: max_i |g_i - o_i| / max(|o_i|, rms(o)) <= 1e-4
+  * bf16-operand paths: max abs <= 2e-2 on unit-scale activations (oracle with bf16 operand emulation)
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import graphs as og
+from oracle import te
+from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+from paper_conf_asplos_xiazswwyfc24_b200.session import session
+
+pytestmark = pytest.mark.gpu
+
+
+def rel_err(g, o):
+    o = np.asarray(o, np.float64)
+    g = np.asarray(g, np.float64)
+    rms = np.sqrt(np.mean(o * o)) + 1e-30
+    return float(np.max(np.abs(g - o) / np.maximum(np.abs(o), rms)))
+
+
+def run(graph, feed, outs, flags=0):
+    plan = graph.partition(L.device_query(0), flags)
+    s = session(graph, plan, feed, outs)
+    s.run()
+    return [s.result(o) for o in outs], plan
+
+
+def _gemm_graph(M_, N, K, relu_a, prec=L.BF16):
+    g = L.Graph()
+    X = g.placeholder((M_, K), L.F32, const=False)
+    W = g.placeholder((N, K), L.BF16 if prec == L.BF16 else L.F32)
+    A = g.ew("relu", X) if relu_a else X
+    Y = g.matmul(A, W, True, prec)
+    g.mark_output(Y)
+    return g, X, W, Y
+
+
+@pytest.mark.parametrize("M_,N,K,relu_a", [(128, 192, 256, False), (128, 192, 256, True), (128, 64, 64, True),
+                                           (200, 128, 128, True), (128, 2304, 768, True)])
+@pytest.mark.parametrize("flags", [0, L.FLAG_UNFUSED])
+def test_tc_gemm_integer_bit_exact(M_, N, K, relu_a, flags):
+    g, X, W, Y = _gemm_graph(M_, N, K, relu_a)
+    x = synth.small_ints(11, (M_, K))
+    w = synth.small_ints(12, (N, K), dtype="bf16")
+    (y,), plan = run(g, {X: x, W: w}, [Y], flags)
+    a = np.maximum(x, 0) if relu_a else x
+    ref = a.astype(np.float64) @ w.astype(np.float64).T
+    assert "GEMM_TC" in plan.describe()
+    assert np.array_equal(y, ref), plan.describe()
+
+
+def test_fig2_fp32_simt():
+    spec, ids = og.fig2()
+    ins = synth.spec_inputs(spec, 3)
+    g, pids = M.fig2()
+    (y,), _ = run(g, {i: v for i, v in ins.items()}, [pids["TE4"]])
+    ref = te.evaluate(spec, ins)[ids["TE4"]]
+    assert rel_err(y, ref) <= 1e-4
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_random_programs_generic_path(seed):
+    spec = synth.random_spec(seed, n_ops=20)
+    ins = synth.spec_inputs(spec, seed)
+    g = M.from_spec(spec)
+    ref = te.evaluate(spec, ins)
+    for flags in (0, L.FLAG_UNFUSED, L.FLAG_NO_GLOBAL_SYNC):
+        outs, plan = run(g, ins, spec["outputs"], flags)
+        for o, y in zip(spec["outputs"], outs):
+            assert rel_err(y, ref[o]) <= 1e-4, (flags, plan.describe())
+
+
+@pytest.mark.parametrize("flags", [0, L.FLAG_UNFUSED, L.FLAG_NO_LN_REWRITE, L.FLAG_NO_VERTICAL])
+def test_bert_tiny_fp32(flags):
+    cfg = synth.BERT_TINY
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    ref = te.evaluate(spec, og.bert_feed(X, plist, x, w))[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    (out,), plan = run(g, og.bert_feed(gX, gpl, x, w), [gy], flags)
+    assert rel_err(out, ref) <= 1e-4, plan.describe()
+
+
+@pytest.mark.parametrize("layers,flags", [(1, 0), (1, L.FLAG_UNFUSED), (12, 0)])
+def test_bert_base_bf16(layers, flags):
+    cfg = dict(synth.BERT_BASE, layers=layers)
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    feed = og.bert_feed(X, plist, x, w)
+    emu = te.evaluate(spec, feed, bf16_operands=True)[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    (out,), plan = run(g, og.bert_feed(gX, gpl, x, w), [gy], flags)
+    err = float(np.abs(out - emu).max())
+    assert err <= 2e-2, (err, plan.describe())
+    if layers == 1:
+        exact = te.evaluate(spec, feed)[y]
+        assert float(np.abs(out - exact).max()) <= 2e-2
+
+
+def test_mmoe():
+    cfg = synth.MMOE_CFG
+    p = synth.mmoe_params(cfg)
+    x = synth.mmoe_input(cfg)
+    spec, names, outs = og.mmoe(cfg)
+    feed = {names[k]: v for k, v in p.items()}
+    feed[names["x"]] = x
+    ref = te.evaluate(spec, feed)
+    g, gn, gouts = M.mmoe(cfg)
+    gfeed = {gn[k]: v for k, v in p.items()}
+    gfeed[gn["x"]] = x
+    res, plan = run(g, gfeed, gouts)
+    for o, r in zip(outs, res):
+        assert rel_err(r, ref[o]) <= 1e-4
+
+
+def test_lstm_small_fp32():
+    cfg = dict(synth.LSTM_CFG, steps=5, layers=3, hidden=64, input=64, w_dtype="f32")
+    x = synth.lstm_input(cfg)
+    ps = synth.lstm_params(cfg)
+    spec, names, top, hs, cs = og.lstm(cfg)
+
+    def feed_for(nm):
+        f = {nm["X"]: x}
+        for n, p in enumerate(ps):
+            f[nm[f"W{n}"]], f[nm[f"U{n}"]] = p["W"], p["U"]
+            f[nm[f"bih{n}"]], f[nm[f"bhh{n}"]] = p["b_ih"], p["b_hh"]
+            f[nm[f"h0_{n}"]] = np.zeros((1, cfg["hidden"]), np.float32)
+            f[nm[f"c0_{n}"]] = np.zeros((1, cfg["hidden"]), np.float32)
+        return f
+
+    ref = te.evaluate(spec, feed_for(names))
+    g, gn, gtop, ghs, gcs = M.lstm(cfg)
+    res, plan = run(g, feed_for(gn), gtop)
+    got = np.concatenate(res)
+    want = np.concatenate([ref[t] for t in top])
+    assert rel_err(got, want) <= 1e-4
