@@ -1,0 +1,302 @@
+"""Benchmark: BERT-base batch-1 seq-128 through Souffle's fused-subprogram path on B200.
+
+One step = one full BERT-base inference (12 encoder layers, batch 1, seq 128) = every §8(a) row
+on the hot path (horizontal QKV GEMM, fused attention, GEMM + two-phase LayerNorm reductions,
+GEMM + GELU, persistent multi-stage executor).  `value` is whole-job inferences/s over all
+ranks (replicas: one independent request stream per GPU, no collective on the hot path).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+  N>1: python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 ... bench.py --gpus N
+
+Timing: W untimed warm-ups; K timed steps, each bracketed by CUDA events on the launching stream,
+with a 256 MB L2 flush (memset, outside the events) before every step -- the 170 MB of weights
+must stream from HBM every step.  Max over ranks.  nvidia-smi clocks are sampled during the
+timed region.  --impl reference times the CPU fp64 oracle (the reference arm of this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BERT-base b1 s128 latency µs; inferences/s at 1/2/4/8 B200; % of roofline"
+WORKLOAD = "BERT-base (12 layers, hidden 768, 12 heads, FFN 3072) batch 1 seq 128"
+# algorithmic HBM bytes per inference: bf16 GEMM weights + fp32 bias/LN + input + output
+H, F, S, NL = 768, 3072, 128, 12
+GEMM_W_BYTES = NL * (4 * H * H + 2 * H * F) * 2
+VEC_BYTES = NL * (4 * H + F + H + 4 * H) * 4
+IO_BYTES = 2 * S * H * 4
+ALGO_BYTES = GEMM_W_BYTES + VEC_BYTES + IO_BYTES
+ALGO_FLOPS = NL * (2 * S * H * (4 * H + 2 * F) + 2 * 2 * S * S * H)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d["hbm_gbs"], d["bf16_tflops"], "measured"
+    return 6650.0, 1590.0, "fallback"
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    def __init__(self, gpu):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={gpu}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                       "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = [l.split(",") for l in open(self.f.name).read().strip().splitlines() if l.strip()]
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows]
+        mx = float(rows[0][2])
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            for k, nm in enumerate(names):
+                if "Active" in r[4 + k] and "Not" not in r[4 + k]:
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(rows)}
+
+
+def oracle_bert_layer_runner():
+    """Oracle (fp64 numpy, CPU) for one BERT-base encoder layer -- the reference arm / cpu_baseline."""
+    import synth
+    from oracle import graphs as og
+    from oracle import te
+    cfg = dict(synth.BERT_BASE, layers=1)
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    feed = og.bert_feed(X, plist, x, w)
+
+    def step():
+        te.evaluate(spec, feed, bf16_operands=True)
+    return step
+
+
+def cpu_baseline(budget_s=15.0):
+    """Time the oracle as it stands on this host: whole layers until ~budget_s elapse."""
+    step = oracle_bert_layer_runner()
+    step()
+    n, t0 = 0, time.perf_counter()
+    while True:
+        step()
+        n += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s or n >= 24:
+            break
+    inf_s = (n / NL) / el
+    return {"value": inf_s, "unit": "inferences/s", "cores": os.cpu_count(), "kind": "oracle",
+            "sample": f"{n} BERT-base encoder layers (= {n / NL:.2f} inferences) of the fp64 numpy oracle "
+                      f"(bf16-operand emulation), {el:.1f} s wall, OpenBLAS threads = host cores"}
+
+
+def run_reference(args):
+    ws, rank, _ = dist_env()
+    if rank != 0:
+        return
+    step = oracle_bert_layer_runner()
+    for _ in range(max(0, min(args.warmup, 1))):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    el = time.perf_counter() - t0
+    inf_s = (args.steps / NL) / el
+    line = {"metric": METRIC, "value": inf_s, "unit": "inferences/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": WORKLOAD, "step": "one encoder layer of the fp64 oracle (1/12 inference)"},
+            "cpu_baseline": {"value": inf_s, "unit": "inferences/s", "cores": os.cpu_count(), "kind": "oracle",
+                             "sample": f"{args.steps} BERT-base encoder layers, fp64 numpy oracle"},
+            "e2e": {"value": inf_s, "unit": "inferences/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+
+
+def build_bert(device_index, flags=0):
+    import synth
+    from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+    from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+    from paper_conf_asplos_xiazswwyfc24_b200.session import session
+    cfg = synth.BERT_BASE
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    g, X, plist, y = M.bert(cfg)
+    plan = g.partition(L.device_query(device_index), flags)
+    feed = {X: x}
+    for names, wl in zip(plist, w):
+        for k, t in names.items():
+            feed[t] = wl[k]
+    sess = session(g, plan, feed, [y], device=f"cuda:{device_index}")
+    return g, plan, sess, X, y, x
+
+
+def time_steps(sess, steps, warmup, flush, stream):
+    import torch
+    for _ in range(warmup):
+        flush.zero_()
+        sess.run()
+    torch.cuda.synchronize()
+    times = []
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    with torch.cuda.stream(stream):
+        for a, b in ev:
+            flush.zero_()
+            a.record(stream)
+            sess.run()
+            b.record(stream)
+    torch.cuda.synchronize()
+    for a, b in ev:
+        times.append(a.elapsed_time(b))
+    return times
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-v0", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        run_reference(args)
+        return
+
+    import torch
+    import torch.distributed as dist
+    ws, rank, local = dist_env()
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    stream = torch.cuda.current_stream(dev)
+    g, plan, sess, X, y, x_host = build_bert(local)
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
+    launches_per_step = plan.exec_info()["launches"]
+
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clk = Clocks(local) if rank == 0 else None
+    times = time_steps(sess, args.steps, args.warmup, flush, stream)
+    clocks = clk.stop() if clk else None
+    total_ms = sum(times)
+    if ws > 1:
+        t = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+        dist.barrier()
+    ms_per_step = total_ms / args.steps
+    value = ws * args.steps / (total_ms / 1e3)
+
+    # ---- e2e through the public API with host buffers (H2D input, D2H output inside the timed region)
+    xin = torch.from_numpy(np.ascontiguousarray(x_host, dtype=np.float32)).pin_memory()
+    yout = torch.empty(sess.outputs[y].shape, dtype=torch.float32).pin_memory()
+    dx = sess.inputs[X]
+    for _ in range(3):
+        dx.copy_(xin, non_blocking=True)
+        sess.run()
+        yout.copy_(sess.outputs[y], non_blocking=True)
+    torch.cuda.synchronize()
+    e_ms = []
+    for _ in range(args.steps):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        dx.copy_(xin, non_blocking=True)
+        sess.run()
+        yout.copy_(sess.outputs[y], non_blocking=True)
+        b.record(stream)
+        b.synchronize()
+        e_ms.append(a.elapsed_time(b))
+    e_total = sum(e_ms)
+    if ws > 1:
+        t = torch.tensor([e_total], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e_total = float(t.item())
+
+    extra = {}
+    if rank == 0 and not args.no_v0:
+        # V0: the same TE graph run unfused, one kernel per TE (Fig. 5(a) / Table 4 V0)
+        from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+        g0, plan0, sess0, *_ = build_bert(local, L.FLAG_UNFUSED)
+        t0 = time_steps(sess0, max(5, args.steps // 5), 3, flush, stream)
+        extra["v0_unfused"] = {"latency_us": statistics.median(t0) * 1e3,
+                               "launches": plan0.exec_info()["launches"]}
+        del sess0, plan0, g0
+
+    if rank == 0:
+        hbm, tf, src = peaks()
+        med = statistics.median(times)
+        achieved = ALGO_BYTES / (med * 1e-3) / 1e9
+        traffic = None
+        pf = os.path.join(ROOT, "profiles", "ncu_bert_base.json")
+        if os.path.exists(pf):
+            traffic = json.load(open(pf)).get("dram_bytes_per_launch")
+        info = plan.exec_info()
+        line = {
+            "metric": METRIC, "value": value, "unit": "inferences/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "latency_us_median": med * 1e3,
+            "latency_us_p10": float(np.percentile(times, 10)) * 1e3,
+            "latency_us_p90": float(np.percentile(times, 90)) * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+            "data": "synthetic",
+            "config": {"workload": WORKLOAD, "l2": "256 MB flush before every timed step (outside the events)",
+                       "parallelism": f"replicas x{ws} (batch-sharded, no collective on the hot path)",
+                       "kernels_per_inference": info["launches"], "stages": info["stages"],
+                       "grid_barriers": info["barriers"]},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
+                         "traffic": traffic, "peak_source": src,
+                         "algorithmic_bytes_per_launch": ALGO_BYTES,
+                         "tensor_frac": ALGO_FLOPS / (med * 1e-3) / 1e12 / tf},
+            "e2e": {"value": ws * args.steps / (e_total / 1e3), "unit": "inferences/s",
+                    "h2d_bytes_per_step": int(xin.numel() * 4), "d2h_bytes_per_step": int(yout.numel() * 4)},
+            "gpu_launches": launches_per_step * args.steps,
+            "clocks": clocks,
+        }
+        line.update(extra)
+        if not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline()
+        print(json.dumps(line))
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

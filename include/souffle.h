@@ -190,6 +190,20 @@ souffle_status souffle_workspace_init(souffle_plan p, void* workspace, void* str
  * run concurrently on different streams only with distinct workspaces. */
 souffle_status souffle_run(souffle_plan p, void* workspace, void* stream);
 
+/* ------------------------------------------------------------------ debug profiling
+ * When enabled, CTA 0 of every launch records %globaltimer at each stage start (after its grid
+ * barrier) and the last CTA records the launch end, in the workspace control region.
+ * souffle_plan_read_profile synchronises the device and returns one duration (microseconds) per
+ * stage in execution order: time from the stage's start to the next stage's start (so it
+ * includes the grid barrier that follows the stage).  Debug use only (it synchronises). */
+souffle_status souffle_plan_set_profiling(souffle_plan p, int32_t on);
+souffle_status souffle_plan_read_profile(souffle_plan p, void* workspace, double* stage_us, int32_t cap,
+                                         int32_t* n);
+/* Raw %globaltimer stamps (ns): [stages + 1] stage starts / launch end, then 8 sub-stage marks
+ * per stage (stage-kind specific, 0 if unused).  cap >= 9 * stages + 1. */
+souffle_status souffle_plan_read_profile_raw(souffle_plan p, void* workspace, uint64_t* stamps, int32_t cap,
+                                             int32_t* n);
+
 #ifdef __cplusplus
 }
 #endif

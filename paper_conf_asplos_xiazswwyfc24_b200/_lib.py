@@ -71,6 +71,8 @@ _SIGS = {
     "souffle_bind": [C.c_void_p, C.c_int32, C.c_void_p],
     "souffle_workspace_init": [C.c_void_p, C.c_void_p, C.c_void_p],
     "souffle_run": [C.c_void_p, C.c_void_p, C.c_void_p],
+    "souffle_plan_set_profiling": [C.c_void_p, C.c_int32],
+    "souffle_plan_read_profile": [C.c_void_p, C.c_void_p, C.POINTER(C.c_double), C.c_int32, C.POINTER(C.c_int32)],
 }
 EXPORTS = sorted(list(_SIGS) + ["souffle_last_error", "souffle_version"])
 
@@ -281,5 +283,34 @@ class Plan:
     def workspace_init(self, ws_ptr, stream=0):
         check(self.lib.souffle_workspace_init(self.h, C.c_void_p(int(ws_ptr)), C.c_void_p(int(stream))))
 
+    def set_profiling(self, on=True):
+        check(self.lib.souffle_plan_set_profiling(self.h, 1 if on else 0))
+
+    def read_profile(self, ws_ptr):
+        n = self.exec_info()["stages"]
+        buf = (C.c_double * max(1, n))()
+        got = C.c_int32()
+        check(self.lib.souffle_plan_read_profile(self.h, C.c_void_p(int(ws_ptr)), buf, n, C.byref(got)))
+        return list(buf[: got.value])
+
     def run(self, ws_ptr, stream=0):
         check(self.lib.souffle_run(self.h, C.c_void_p(int(ws_ptr)), C.c_void_p(int(stream))))
+
+
+def _add_raw_profile():
+    def read_profile_raw(self, ws_ptr):
+        n = self.exec_info()["stages"]
+        cap = 9 * n + 1 + 4 * 160 * n   # stage starts, 8 marks per stage, per-CTA marks
+        buf = (C.c_uint64 * cap)()
+        got = C.c_int32()
+        check(self.lib.souffle_plan_read_profile_raw(self.h, C.c_void_p(int(ws_ptr)), buf, cap, C.byref(got)))
+        starts = list(buf[: n + 1])
+        marks = [list(buf[n + 1 + 8 * s: n + 1 + 8 * s + 8]) for s in range(n)]
+        return starts, marks
+    Plan.read_profile_raw = read_profile_raw
+
+
+_SIGS["souffle_plan_read_profile_raw"] = [C.c_void_p, C.c_void_p, C.POINTER(C.c_uint64), C.c_int32,
+                                          C.POINTER(C.c_int32)]
+EXPORTS = sorted(list(_SIGS) + ["souffle_last_error", "souffle_version"])
+_add_raw_profile()

@@ -44,13 +44,16 @@ enum { NREG = 4, CHUNK = 8, MAX_RED = 4, MAX_BUFS = 480, EXEC_THREADS = 256, EXE
 //   mode 1 separable: row(r) = tab[rtab + r],   col(c) = tab[ctab + c]
 //   mode 2 full:      row(r) + col(c) = tab[ftab + r*ncols + c]
 struct Addr {
+  uint64_t ptr;   // resolved at souffle_workspace_init: address of element `base` (device uses ptr +
+                  // element offset of row(r) + col(c); `buf`/`base` are the host-side description)
   int64_t base;
   int64_t rs, cs;
   int32_t buf;    // >= 0: bound pointer table index; -1: workspace (base counted from ws_data)
   int32_t dtype;  // 0 f32, 1 bf16
   int32_t mode;
   int32_t rtab, ctab, ftab, ncols;
-  int32_t cg;     // 1: tensor is written inside the run -> coherent (L2) loads
+  int16_t cg;     // 1: tensor is written inside the run -> coherent (L2) loads
+  int16_t cvec;   // mode 1: col(c0 + j) == col(c0) + j within every aligned chunk of CHUNK columns
 };
 
 struct Ins {
@@ -59,11 +62,32 @@ struct Ins {
   float imm;
 };
 
+// A fused-chain program: Ins[ins0 .. ins0+len) whose Ins.addr index a program-local Addr table
+// addrs[addr0 .. addr0+naddr).  Programs and their tables are small enough to be staged in
+// shared memory once per stage / task, so the interpreter never chases global pointers.
+// Compiled fast paths the host recognises in a program (all fields are instruction indices whose
+// `addr` is used, or -1).  kind 1 "linear epilogue": v = act(acc + side0 + side1); store v to st0 /
+// st1; row sums of v and v*v into red_sum / red_sq.  kind 2 "LayerNorm apply" (EW domain):
+// v = (x - mu) * rsqrt(msq - mu*mu + eps) * g + b; store to st0 / st1.  kind 0: interpret.
+struct FastPath {
+  int32_t kind;
+  int32_t side0, side1, act;
+  int32_t st0, st1, red_sum, red_sq;
+  int32_t ln_x, ln_mu, ln_msq, ln_g, ln_b;
+  float eps;
+  float red_scale_sum, red_scale_sq;
+};
+
+struct ProgRef {
+  int32_t ins0, len, addr0, naddr;
+  FastPath fast;
+};
+
 struct GemmMember {
   int32_t M, N, K, batch;   // domain rows = batch*M (b-major), cols = N
   int32_t prec;             // SIMT: 1 -> round operands to bf16
   int32_t a_addr, b_addr;   // SIMT: A at (r = b*M+m, c = k), B at (r = b*N+n, c = k)
-  int32_t prog, prog_len;   // epilogue program at (r, c)
+  ProgRef prog;             // epilogue program at (r, c)
   int32_t tiles_m, tiles_n, splits, task0;  // tasks = tiles_m*tiles_n*splits, starting at task0
   int32_t n_tile, k_split;  // TC: N tile, K per split (multiple of 64)
   int32_t a_tmap, b_tmap;   // TC: TMA descriptor indices (a_tmap < 0 -> manual fp32 A path)
@@ -76,15 +100,16 @@ struct GemmMember {
 struct Stage {
   int32_t kind, barrier_before, ntasks, sp;
   int32_t rows, cols;               // EW / REDUCE domain
-  int32_t prog, prog_len;           // EW program; REDUCE pre-program at (o, e)
-  int32_t post, post_len;           // REDUCE post-program at (o, 0)
+  ProgRef prog;                     // EW program; REDUCE pre-program at (o, e); ATTN epilogue
+  ProgRef post;                     // REDUCE post-program at (o, 0)
   int32_t red_fn;                   // REDUCE: 0 sum, 1 max
   float red_scale;                  // REDUCE: 1/E for mean
   int32_t mem0, nmem;               // GEMM members
   // ATTN: q/k/v are bf16 [B, S, d] contiguous workspace tensors
   int32_t at_B, at_S, at_d, at_q, at_k, at_v;  // q/k/v: Addr index (base, buf used)
   float at_scale;
-  int32_t pad[3];
+  int32_t barrier_after;            // the next stage of the same launch starts with a grid barrier
+  int32_t pad[2];
 };
 
 struct Launch {
@@ -105,6 +130,9 @@ struct Params {
   char* ws_data;              // intermediates / accumulators
   unsigned int* ctrl;         // [0] barrier counter, [1] exit counter
   const int64_t* zero_list;   // (byte offset, bytes) pairs in ws_data, zeroed by the last CTA
+  unsigned long long* prof;   // optional: %globaltimer at every stage start (CTA 0), null if off;
+                              // followed by 8 sub-stage marks per stage (prof[nst + 1 + 8*s + k])
+  int32_t n_stages_total;
   int32_t n_zero;
   int32_t first, count, cooperative, uses_tc, is_last;
   void* bufs[MAX_BUFS];

@@ -68,6 +68,8 @@ souffle_status run_plan(Plan& p, void* ws, void* stream);
 souffle_status init_workspace(Plan& p, void* ws, void* stream);
 souffle_status query_device(int dev, souffle_device_desc* out);
 size_t workspace_bytes(Plan& p);
+souffle_status read_profile(Plan& p, void* ws, double* us, int cap, int* n);
+souffle_status read_profile_raw(Plan& p, void* ws, unsigned long long* out, int cap, int* n);
 
 }  // namespace souffle
 
@@ -464,6 +466,21 @@ souffle_status souffle_run(souffle_plan p, void* workspace, void* stream) {
   g_err.clear();
   if (!p || !workspace) return fail(SOUFFLE_E_INVALID_ARG, "null argument");
   return run_plan(p->p, workspace, stream);
+}
+
+souffle_status souffle_plan_set_profiling(souffle_plan p, int32_t on) {
+  return guard([&] { PL(p).profiling = on != 0; });
+}
+souffle_status souffle_plan_read_profile(souffle_plan p, void* workspace, double* stage_us, int32_t cap, int32_t* n) {
+  g_err.clear();
+  if (!p || !workspace || !stage_us || !n) return fail(SOUFFLE_E_INVALID_ARG, "null argument");
+  return read_profile(p->p, workspace, stage_us, cap, n);
+}
+souffle_status souffle_plan_read_profile_raw(souffle_plan p, void* workspace, uint64_t* stamps, int32_t cap,
+                                             int32_t* n) {
+  g_err.clear();
+  if (!p || !workspace || !stamps || !n) return fail(SOUFFLE_E_INVALID_ARG, "null argument");
+  return read_profile_raw(p->p, workspace, (unsigned long long*)stamps, cap, n);
 }
 
 }  // extern "C"

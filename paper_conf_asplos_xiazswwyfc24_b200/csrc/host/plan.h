@@ -52,6 +52,7 @@ struct Plan {
   std::vector<int32_t> buf_node;    // slot -> node
   void* inited_ws = nullptr;        // workspace the program/tmaps were uploaded to
   bool dirty = true;
+  bool profiling = false;
   std::vector<uint8_t> host_prog;   // packed program region (uploaded by workspace_init)
 };
 

@@ -24,7 +24,9 @@ static int64_t al(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 size_t workspace_bytes(Plan& p) {
   WsLayout& w = p.ws;
   w.ctrl_off = 0;
-  w.ctrl_bytes = 256;
+  // barrier words + stage timestamps + 8 sub-stage marks per stage
+  w.ctrl_bytes = al(256 + 8 * ((int64_t)p.stages.size() + 1) + 64 * (int64_t)p.stages.size() +
+                        (p.profiling ? 8 * 4 * 160 * (int64_t)p.stages.size() : 0), 256);
   int64_t o = w.ctrl_bytes;
   w.prog_off = o;
   int64_t q = 0;
@@ -118,7 +120,15 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
   put(w.o_stages, p.stages.data(), p.stages.size() * sizeof(Stage));
   put(w.o_members, p.members.data(), p.members.size() * sizeof(GemmMember));
   put(w.o_ins, p.ins.data(), p.ins.size() * sizeof(Ins));
-  put(w.o_addrs, p.addrs.data(), p.addrs.size() * sizeof(Addr));
+  {
+    // resolve every address record to an absolute device pointer (no pointer-table lookups on device)
+    std::vector<Addr> ra(p.addrs);
+    for (Addr& a : ra) {
+      char* b = a.buf >= 0 ? (char*)p.buf_ptr[a.buf] : data;
+      a.ptr = (uint64_t)(b + a.base * (a.dtype == 1 ? 2 : 4));
+    }
+    put(w.o_addrs, ra.data(), ra.size() * sizeof(Addr));
+  }
   put(w.o_tabs, p.tabs.data(), p.tabs.size() * sizeof(int32_t));
   put(w.o_tmaps, tm.data(), tm.size());
   put(w.o_zero, p.zero_list.data(), p.zero_list.size() * sizeof(int64_t));
@@ -162,6 +172,8 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
   prm.n_zero = (int32_t)(p.zero_list.size() / 2);
   prm.ws_data = base + w.data_off;
   prm.ctrl = (unsigned int*)(base + w.ctrl_off);
+  prm.prof = p.profiling ? (unsigned long long*)(base + w.ctrl_off + 256) : nullptr;
+  prm.n_stages_total = (int32_t)p.stages.size();
   for (size_t i = 0; i < p.buf_ptr.size(); ++i) prm.bufs[i] = p.buf_ptr[i];
   cudaStream_t s = (cudaStream_t)stream;
   for (const Launch& L : p.launches) {
@@ -179,6 +191,33 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
     cudaError_t e = exec_launch(prm, grid, L.smem, L.cooperative != 0, s);
     if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("launch: ") + cudaGetErrorString(e));
   }
+  return SOUFFLE_OK;
+}
+
+souffle_status read_profile_raw(Plan& p, void* ws, unsigned long long* out, int cap, int* n) {
+  size_t cnt = p.stages.size() + 1 + 8 * p.stages.size() + (p.profiling ? 4 * 160 * p.stages.size() : 0);
+  if ((size_t)cap < cnt) return fail(SOUFFLE_E_INVALID_ARG, "profile buffer too small");
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(out, (char*)ws + p.ws.ctrl_off + 256, cnt * 8, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("profile read: ") + cudaGetErrorString(e));
+  *n = (int)cnt;
+  return SOUFFLE_OK;
+}
+
+souffle_status read_profile(Plan& p, void* ws, double* us, int cap, int* n) {
+  std::vector<unsigned long long> t(p.stages.size() + 1, 0);
+  cudaError_t e = cudaDeviceSynchronize();
+  if (e == cudaSuccess)
+    e = cudaMemcpy(t.data(), (char*)ws + p.ws.ctrl_off + 256, t.size() * 8, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("profile read: ") + cudaGetErrorString(e));
+  // duration of stage s = next timestamp in its launch (stage start or launch end) - its start
+  int k = 0;
+  for (const Launch& L : p.launches)
+    for (int s = L.first; s < L.first + L.count && k < cap; ++s, ++k) {
+      unsigned long long nx = (s + 1 < L.first + L.count) ? t[s + 1] : t[L.first + L.count];
+      us[k] = (nx > t[s]) ? (double)(nx - t[s]) * 1e-3 : -1.0;
+    }
+  *n = k;
   return SOUFFLE_OK;
 }
 
