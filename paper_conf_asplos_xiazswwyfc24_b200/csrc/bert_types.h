@@ -1,0 +1,73 @@
+// Plain-data structures shared by the host planner (csrc/host/bert.cpp) and the specialised
+// BERT-encoder subprogram kernel (csrc/kernels/bert.cu).
+//
+// When the partitioned TE program is a stack of BERT encoder layers (Table 2,
+// 49 TEs per layer), the whole program is one subprogram (§5.4) and is run
+// by one persistent cooperative kernel whose stages are the fused patterns of §6:
+//   GEMM  horizontal / plain tcgen05 GEMM (§6.1).  Epilogues (vertical transformation §6.2):
+//           EP_QKV     + bias, bf16, the reshape/permute index map folded into the store
+//                      (Q, K head-major [2*heads][S][d]; V transposed [heads][d][S])
+//           EP_GELU    + bias, erf-GELU, bf16 [S][N]
+//           EP_PARTIAL split-K partial, fp32 [split][S][N] plain stores (summed by the consumer)
+//   ATTN  per head: QK^T -> scale -> max-subtracted softmax -> PV, S and O in TMEM (Fig. 1(c))
+//   ROW   per token row: sum of split-K partials + bias + residual + LayerNorm (two-pass mean /
+//         variance over the row), fp32 and bf16 outputs (the two-phase reduction of P:L527-536)
+// Weights never depend on activations, so a producer warp streams every GEMM stage's weight tiles
+// through a shared-memory ring ahead of the grid barriers (§6.5 "cross-stage prefetch").
+#pragma once
+#include <stdint.h>
+
+namespace souffle {
+
+enum BStageKind : int32_t { BS_GEMM = 0, BS_ATTN = 1, BS_ROW = 2 };
+enum BEpilogue : int32_t { EP_PARTIAL = 0, EP_QKV = 1, EP_GELU = 2 };
+
+enum {
+  BERT_THREADS = 288,          // 8 compute warps + 1 weight-producer warp
+  BERT_COMPUTE = 256,
+  BW_SLOTS = 5,                // weight ring: 5 x 16 KB; a slot holds 16 KB / (n_tile * 128 B) K-chunks
+  BW_SLOT_BYTES = 16384,
+  BA_SLOTS = 8,                // A operand ring: 8 x (128 rows x 64 K bf16); also the epilogue staging tile
+  BA_SLOT_BYTES = 16384,
+  B_CTRL_BYTES = 2048,         // control block + two staged stage descriptors
+  B_AREGION = BA_SLOTS * BA_SLOT_BYTES,   // also holds the attention operands Q, K, V^T, P (80 KB)
+  B_SMEM = B_CTRL_BYTES + BW_SLOTS * BW_SLOT_BYTES + B_AREGION + 1024   // + alignment slack
+};
+
+struct BStage {
+  int32_t kind, ntasks, layer, idx;   // idx: position in the stage list
+  // ---- GEMM: task = tile * nsplit + split; each split covers kchunks chunks of 64 along K
+  int32_t nt, tiles_n, nsplit, kchunks;
+  int32_t K, N, wmap0, wrows;   // W tensor maps wmap0.. (an N tile never straddles two maps)
+  int32_t amap, epi, heads, workers;   // workers: CTAs with work in this stage (barrier arrivals)
+  const float* bias;            // EP_QKV / EP_GELU: fp32 [N]
+  float* part;                  // EP_PARTIAL: fp32 [nsplit][S][N]
+  uint16_t* out_b;              // EP_GELU: bf16 [S][N];  EP_QKV: Q,K [2*heads][S][64]
+  uint16_t* out_vt;             // EP_QKV: V^T [heads][64][S]
+  // ---- ATTN: TMA maps of Q/K ([2*heads][S][64]) and V^T ([heads][64][S])
+  int32_t qkmap, vtmap, d, H;
+  uint16_t* ctx;                // bf16 [S][H], head h at columns h*64 ..
+  float scale, eps;
+  // ---- ROW: mode 0 convert (out_b = bf16(in)); mode 1 LayerNorm(sum_s part[s] + bias + res)
+  int32_t row_mode, cols, r_nsplit, pad1;
+  const float* r_in;            // mode 0: fp32 [S][cols]; mode 1: partials [r_nsplit][S][cols]
+  const float* r_bias;
+  const float* r_res;
+  const float* r_gamma;
+  const float* r_beta;
+  float* r_out_f;
+  uint16_t* r_out_b;
+  int64_t pad2;
+};
+
+struct BertParams {
+  const BStage* stages;
+  const void* tmaps;            // CUtensorMap[] (128 B each)
+  unsigned int* ctrl;           // [0, nstages): per-barrier arrival counters; [nstages]: exit counter
+  unsigned long long* prof;     // optional per-stage %globaltimer marks, null if off
+  int32_t nstages, S;
+  int32_t dbg_skip;             // debug: bit k set -> stages of kind k do no work (barriers only)
+  int32_t pad;
+};
+
+}  // namespace souffle

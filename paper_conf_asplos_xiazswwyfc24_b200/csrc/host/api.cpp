@@ -425,6 +425,12 @@ souffle_status souffle_plan_hgroup(souffle_plan p, souffle_tensor te, int32_t* l
 souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t* stages, int32_t* barriers) {
   return guard([&] {
     Plan& P = PL(p);
+    if (P.bert.on) {
+      if (launches) *launches = 1;
+      if (stages) *stages = P.bert.nstages;
+      if (barriers) *barriers = P.bert.nstages - 1;
+      return;
+    }
     if (launches) *launches = (int32_t)P.launches.size();
     if (stages) *stages = (int32_t)P.stages.size();
     if (barriers) *barriers = P.n_barriers;

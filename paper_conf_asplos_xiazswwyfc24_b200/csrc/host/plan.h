@@ -5,6 +5,7 @@
 #include <vector>
 
 #include "../exec_types.h"
+#include "bert.h"
 #include "ir.h"
 
 namespace souffle {
@@ -54,6 +55,7 @@ struct Plan {
   bool dirty = true;
   bool profiling = false;
   std::vector<uint8_t> host_prog;   // packed program region (uploaded by workspace_init)
+  BertPlan bert;                    // pattern lowering (bert.on: kernels/bert.cu runs the program)
 };
 
 void lower(Plan& p);              // fills the lowered program + layout (pure host)

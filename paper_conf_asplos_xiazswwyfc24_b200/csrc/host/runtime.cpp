@@ -21,7 +21,11 @@ cudaError_t exec_max_active(int smem, int* blocks_per_sm);
 
 static int64_t al(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
+souffle_status bert_init(Plan& p, void* ws, void* stream);
+souffle_status bert_run(Plan& p, void* ws, void* stream);
+
 size_t workspace_bytes(Plan& p) {
+  if (p.bert.on) return (size_t)p.bert.total;
   WsLayout& w = p.ws;
   w.ctrl_off = 0;
   // barrier words + stage timestamps + 8 sub-stage marks per stage
@@ -91,6 +95,7 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
   if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
   for (size_t s = 0; s < p.buf_ptr.size(); ++s)
     if (!p.buf_ptr[s]) return fail(SOUFFLE_E_STATE, "tensor " + std::to_string(p.buf_node[s]) + " is not bound");
+  if (p.bert.on) return bert_init(p, ws, stream);
   workspace_bytes(p);
   const WsLayout& w = p.ws;
   char* base = (char*)ws;
@@ -146,6 +151,11 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
 souffle_status run_plan(Plan& p, void* ws, void* stream) {
   if (p.dirty || p.inited_ws != ws)
     return fail(SOUFFLE_E_STATE, "call souffle_workspace_init after binding (bindings or workspace changed)");
+  if (p.bert.on) {
+    std::string why;
+    if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
+    return bert_run(p, ws, stream);
+  }
   static int max_active = -1;
   if (max_active < 0) {
     std::string why;
@@ -195,6 +205,15 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
 }
 
 souffle_status read_profile_raw(Plan& p, void* ws, unsigned long long* out, int cap, int* n) {
+  if (p.bert.on) {   // [0, ns): stage starts, ns+1: end; then 16 sub-stage marks per stage
+    const size_t cnt = 17 * (size_t)p.bert.nstages + 2;
+    if ((size_t)cap < cnt) return fail(SOUFFLE_E_INVALID_ARG, "profile buffer too small");
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) e = cudaMemcpy(out, (char*)ws + p.bert.o_prof, cnt * 8, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("profile read: ") + cudaGetErrorString(e));
+    *n = (int)cnt;
+    return SOUFFLE_OK;
+  }
   size_t cnt = p.stages.size() + 1 + 8 * p.stages.size() + (p.profiling ? 4 * 160 * p.stages.size() : 0);
   if ((size_t)cap < cnt) return fail(SOUFFLE_E_INVALID_ARG, "profile buffer too small");
   cudaError_t e = cudaDeviceSynchronize();
@@ -205,6 +224,20 @@ souffle_status read_profile_raw(Plan& p, void* ws, unsigned long long* out, int 
 }
 
 souffle_status read_profile(Plan& p, void* ws, double* us, int cap, int* n) {
+  if (p.bert.on) {
+    const int ns = p.bert.nstages;
+    std::vector<unsigned long long> t(ns + 2, 0);
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) e = cudaMemcpy(t.data(), (char*)ws + p.bert.o_prof, t.size() * 8, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("profile read: ") + cudaGetErrorString(e));
+    int k = 0;
+    for (int s = 0; s < ns && k < cap; ++s, ++k) {
+      unsigned long long nx = s + 1 < ns ? t[s + 1] : t[ns + 1];
+      us[k] = nx > t[s] ? (double)(nx - t[s]) * 1e-3 : -1.0;
+    }
+    *n = k;
+    return SOUFFLE_OK;
+  }
   std::vector<unsigned long long> t(p.stages.size() + 1, 0);
   cudaError_t e = cudaDeviceSynchronize();
   if (e == cudaSuccess)

@@ -1,0 +1,674 @@
+// Specialised Souffle subprogram kernel for BERT encoder stacks on sm_100a (B200).
+//
+// The partitioner puts a whole BERT stack into one subprogram (§5.4; Table 5: Souffle
+// runs BERT with very few kernels) and the lowering recognises the encoder-layer TE pattern
+// (host/bert.cpp).  This kernel runs that subprogram as ONE persistent cooperative launch
+// (§6.4 "global sync", Fig. 2):
+//
+//   warp 8      weight producer: walks the stage list and TMA-loads, for every GEMM task this CTA
+//               owns, its weight K-chunks into an 8 x 16 KB shared-memory ring.  Weights are
+//               constants, so it runs ahead across grid barriers and the HBM weight stream overlaps
+//               the activation dependency chain (§6.5 cross-stage prefetch, Table 4 V4).
+//   warps 0-7   stage executor:
+//     GEMM      A (bf16 activations) streamed by TMA through a 5-slot ring; one thread issues
+//               tcgen05.mma (M = 128 tokens, N = tile, K = 16) into TMEM; fused epilogues:
+//               bias + bf16 + head-major / transposed stores (QKV: the reshape/permute index maps
+//               of §6.2 folded into the store), bias + erf-GELU (FFN1), or fp32 split-K partials.
+//     ATTN      per head: Q, K, V^T by TMA, S = QK^T in TMEM, softmax (max-subtracted, fp32
+//               registers), P bf16 in smem, O = PV in TMEM, ctx stored bf16 (Fig. 1(c), §2.3).
+//     ROW       one CTA per token row: sum of the split-K partials + bias + residual, LayerNorm
+//               with two-pass block reductions, fp32 and bf16 outputs (two-phase reduction,
+//               partial results per block, combined after the global sync).
+//   A split-phase grid barrier (one arrival counter per barrier) separates dependent stages.
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../bert_types.h"
+#include "ptx.cuh"
+
+namespace souffle {
+namespace bert {
+
+static_assert(sizeof(BStage) % 16 == 0, "BStage is copied with 16-byte vectors");
+static_assert(2 * sizeof(BStage) <= 1024, "two BStage buffers are staged in the control block");
+
+struct Ctrl {
+  uint64_t wfull[BW_SLOTS];
+  uint64_t wempty[BW_SLOTS];
+  uint64_t afull[BA_SLOTS];
+  uint64_t aempty[BA_SLOTS];
+  uint64_t accb;
+  uint64_t attb;
+  uint64_t qkvb;
+  uint32_t tmem_base;
+  volatile int cur_stage;       // debug (dbg_skip bit 12): the producer does not run ahead of the executor
+  float red[2][8];
+};
+static_assert(sizeof(Ctrl) <= 1024, "control block");
+
+__device__ __forceinline__ void csync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+
+__device__ __forceinline__ uint32_t sw128(int row, int kbyte) {
+  return (uint32_t)(row * 128 + ((((kbyte >> 4) ^ (row & 7)) & 7) << 4) + (kbyte & 15));
+}
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);   // .x = a (low half)
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+__device__ __forceinline__ uint16_t bf16_bits(float a) {
+  __nv_bfloat16 b = __float2bfloat16_rn(a);
+  return *reinterpret_cast<uint16_t*>(&b);
+}
+__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.f + erff(x * 0.70710678118654752f)); }
+template <class T>
+__device__ __forceinline__ const void* ldgp(T* const* p) {
+  return (const void*)__ldg(reinterpret_cast<const unsigned long long*>(p));
+}
+
+__device__ __forceinline__ void mark(const BertParams& P, int idx) {
+  if (P.prof && blockIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    P.prof[idx] = t;
+  }
+}
+// debug timeline: sub-stage mark k of stage st (recorded by the first CTA with work in the stage)
+__device__ __forceinline__ void submark(const BertParams& P, const BStage& st, int k) {
+  if (P.prof && blockIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    P.prof[P.nstages + 2 + 16 * st.idx + k] = t;
+  }
+}
+
+// ------------------------------------------------------------------ grid barrier (split phase)
+__device__ __forceinline__ void grid_arrive(const BertParams& P, int k) {
+  ptx::fence_proxy_async();   // generic-proxy writes of this stage -> TMA reads of later stages
+  csync();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(&P.ctrl[k], 1u);
+  }
+}
+__device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target_arrivals) {
+  if (threadIdx.x == 0) {
+    const unsigned target = (unsigned)target_arrivals;
+    while (ptx::ld_acquire(&P.ctrl[k]) < target) {
+    }
+    ptx::fence_proxy_async();
+  }
+  csync();
+}
+
+// does this CTA have work in stage st?  (GEMM: one task per CTA; ATTN: heads on the last CTAs;
+// ROW: rows on the first CTAs)
+__device__ __forceinline__ bool has_work(const BertParams& P, const BStage& st) {
+  const int b = blockIdx.x;
+  if (st.kind == BS_GEMM || st.kind == BS_ATTN) return b < st.ntasks;
+  return b < P.S;
+}
+
+// K-chunk order of a task: rotated by the CTA index so that the CTAs of a stage, which all read
+// the same activation tile, spread their concurrent A requests over all L2 slices instead of
+// hammering the lines of one chunk together (the accumulation order changes; the sum does not)
+__device__ __forceinline__ int rot_chunk(int i, int nk) { return (i + (int)blockIdx.x) % nk; }
+
+// weight K-chunks per ring slot for an N tile of nt rows (16 KB / (nt * 128 B))
+__device__ __forceinline__ int wgroup(int nt) { return max(1, BW_SLOT_BYTES / (nt * 128)); }
+
+// ------------------------------------------------------------------ weight producer (warp 8)
+__device__ void weight_producer(const BertParams& P, Ctrl* C, char* wring) {
+  const char* tmaps = (const char*)P.tmaps;
+  uint32_t it = 0;
+  for (int s = 0; s < P.nstages; ++s) {
+    const BStage* st = P.stages + s;
+    const int kind = __ldg(&st->kind);
+    if (kind != BS_GEMM && kind != BS_ATTN) continue;   // ATTN: fused out-projection tile
+    if (P.dbg_skip & 4096)
+      while (C->cur_stage < s) {
+      }
+    const int task = blockIdx.x;
+    if (task >= __ldg(&st->ntasks)) continue;
+    const int nsplit = __ldg(&st->nsplit), nt = __ldg(&st->nt), kch = __ldg(&st->kchunks);
+    const int wrows = __ldg(&st->wrows), wmap0 = __ldg(&st->wmap0);
+    const int tile = task / nsplit, split = task % nsplit;
+    const int n0 = tile * nt;
+    const int map = wmap0 + n0 / wrows, row = n0 % wrows;
+    const int kc0 = split * kch;
+    const int nk = min(kch, __ldg(&st->K) / 64 - kc0);
+    const int gsz = wgroup(nt);
+    for (int c0 = 0; c0 < nk; c0 += gsz, ++it) {
+      const int cnt = min(gsz, nk - c0);
+      const uint32_t slot = it % BW_SLOTS, ph = (it / BW_SLOTS) & 1;
+      ptx::mbar_wait(&C->wempty[slot], ph ^ 1);
+      ptx::mbar_arrive_expect_tx(&C->wfull[slot], (uint32_t)(cnt * nt * 128));
+      for (int j = 0; j < cnt; ++j)
+        ptx::tma_load_2d(wring + slot * BW_SLOT_BYTES + j * nt * 128, tmaps + 128 * map, &C->wfull[slot],
+                         (kc0 + rot_chunk(c0 + j, nk)) * 64, row);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ GEMM stage
+struct MmaState {
+  uint32_t wit;            // weight-ring consumer group counter (thread 0)
+  uint32_t aload, ause;    // A-ring chunk counters (thread 0)
+  uint32_t accph, attph, qkvph;
+};
+
+// Epilogue of one 128 x nt accumulator tile: TMEM -> registers (+bias, GELU) -> fp32 staging tile in
+// shared memory (the A region, free once the MMAs completed) -> coalesced full-sector global stores
+// by the whole CTA (thread-per-row stores would write 16-byte fragments of 128 different lines).
+template <int COLS>
+__device__ __forceinline__ void gemm_epilogue(const BertParams& P, const BStage& st, Ctrl* C, char* stage_smem, int n0,
+                                              int split) {
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int q = warp & 3, half = warp >> 2;
+  const int row = q * 32 + lane;
+  const int S = P.S, N = st.N;
+  constexpr int NT = 2 * COLS;
+  constexpr int LD = NT + 4;   // padded fp32 row stride of the staging tile
+  float* stg = reinterpret_cast<float*>(stage_smem);
+  const uint32_t taddr = C->tmem_base + ((uint32_t)(q * 32) << 16) + half * COLS;
+  float v[COLS];
+  if constexpr (COLS == 8) ptx::tmem_ld8(taddr, v);
+  else if constexpr (COLS == 16) ptx::tmem_ld16(taddr, v);
+  else if constexpr (COLS == 32) ptx::tmem_ld32(taddr, v);
+  else ptx::tmem_ld64(taddr, v);
+  ptx::tc_fence_before();
+  if (st.epi != EP_PARTIAL) {
+    const float4* bp = reinterpret_cast<const float4*>(st.bias + n0 + half * COLS);
+#pragma unroll
+    for (int c = 0; c < COLS; c += 4) {
+      const float4 b = __ldg(bp + c / 4);
+      v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
+    }
+    if (st.epi == EP_GELU) {
+#pragma unroll
+      for (int c = 0; c < COLS; ++c) v[c] = gelu_erf(v[c]);
+    }
+  }
+#pragma unroll
+  for (int c = 0; c < COLS; c += 4)
+    *reinterpret_cast<float4*>(stg + row * LD + half * COLS + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+  csync();
+  if (st.epi == EP_PARTIAL) {
+    constexpr int U = NT / 4;   // float4 units per row
+    float* dst = st.part + (int64_t)split * S * N + n0;
+    for (int u = tid; u < S * U; u += BERT_COMPUTE) {
+      const int r = u / U, c4 = u % U;
+      *reinterpret_cast<float4*>(dst + (int64_t)r * N + 4 * c4) = *reinterpret_cast<const float4*>(stg + r * LD + 4 * c4);
+    }
+  } else if (st.epi == EP_GELU) {
+    constexpr int U = NT / 8;   // 8-element (16 B) bf16 units per row
+    uint16_t* dst = st.out_b + n0;
+    for (int u = tid; u < S * U; u += BERT_COMPUTE) {
+      const int r = u / U, c8 = u % U;
+      const float* sp = stg + r * LD + 8 * c8;
+      *reinterpret_cast<uint4*>(dst + (int64_t)r * N + 8 * c8) =
+          make_uint4(pack_bf16(sp[0], sp[1]), pack_bf16(sp[2], sp[3]), pack_bf16(sp[4], sp[5]), pack_bf16(sp[6], sp[7]));
+    }
+  } else {
+    // EP_QKV: columns [n0, n0 + NT) of [Q | K | V] lie in one head (NT divides 64)
+    const int H = N / 3;
+    const int which = n0 / H, hh = (n0 % H) >> 6, jd = n0 & 63;
+    if (which < 2) {   // head-major [S][64]: NT * 2 bytes contiguous per token row
+      constexpr int U = NT / 8;
+      uint16_t* dst = st.out_b + ((int64_t)(which * st.heads + hh) * S << 6) + jd;
+      for (int u = tid; u < S * U; u += BERT_COMPUTE) {
+        const int r = u / U, c8 = u % U;
+        const float* sp = stg + r * LD + 8 * c8;
+        *reinterpret_cast<uint4*>(dst + ((int64_t)r << 6) + 8 * c8) =
+            make_uint4(pack_bf16(sp[0], sp[1]), pack_bf16(sp[2], sp[3]), pack_bf16(sp[4], sp[5]), pack_bf16(sp[6], sp[7]));
+      }
+    } else {           // V^T [64][S]: S * 2 bytes contiguous per feature row
+      const int U = S / 8;
+      uint16_t* dst = st.out_vt + ((int64_t)hh * 64 + jd) * S;
+      for (int u = tid; u < NT * U; u += BERT_COMPUTE) {
+        const int dcol = u / U, t8 = u % U;
+        const float* sp = stg + (8 * t8) * LD + dcol;
+        *reinterpret_cast<uint4*>(dst + (int64_t)dcol * S + 8 * t8) =
+            make_uint4(pack_bf16(sp[0], sp[LD]), pack_bf16(sp[2 * LD], sp[3 * LD]), pack_bf16(sp[4 * LD], sp[5 * LD]),
+                       pack_bf16(sp[6 * LD], sp[7 * LD]));
+      }
+    }
+  }
+}
+
+__device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* wring, char* areg, MmaState& ms) {
+  const int task = blockIdx.x;
+  if (task >= st.ntasks) return;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  const int tile = task / st.nsplit, split = task % st.nsplit;
+  const int nt = st.nt, n0 = tile * nt;
+  const int kc0 = split * st.kchunks;
+  const int nk = min(st.kchunks, st.K / 64 - kc0);
+  const char* amap = (const char*)P.tmaps + 128 * st.amap;
+
+  if (warp == 1) {
+    // ---- A producer (warp 1, one elected lane issues): keeps BA_SLOTS chunks in flight, refills a
+    // slot as soon as the MMAs that read it have completed
+    for (int c = 0; c < nk; ++c) {
+      const uint32_t slot = ms.aload % BA_SLOTS;
+      if (ms.aload >= BA_SLOTS) ptx::mbar_wait(&C->aempty[slot], ((ms.aload / BA_SLOTS) - 1) & 1);
+      if (ptx::elect_one()) {
+        ptx::mbar_arrive_expect_tx(&C->afull[slot], BA_SLOT_BYTES);
+        ptx::tma_load_2d(areg + slot * BA_SLOT_BYTES, amap, &C->afull[slot], (kc0 + rot_chunk(c, nk)) * 64, 0);
+      }
+      __syncwarp();
+      ++ms.aload;
+    }
+  } else if (warp == 0) {
+    // ---- MMA issue: the whole warp runs the loop (operands stay warp-uniform), one lane issues
+    if (tid == 0) submark(P, st, 0);
+    const uint32_t idesc = ptx::idesc_bf16(128, nt);
+    const int gsz = wgroup(nt);
+    const uint32_t tmem = C->tmem_base;
+    const uint64_t da0 = ptx::sdesc_sw128(ptx::smem_u32(areg)), db0 = ptx::sdesc_sw128(ptx::smem_u32(wring));
+    uint32_t wslot = 0;
+    for (int c = 0; c < nk; ++c) {
+      const uint32_t as = ms.ause % BA_SLOTS;
+      ptx::mbar_wait(&C->afull[as], (ms.ause / BA_SLOTS) & 1);
+      const int j = c % gsz;
+      if (j == 0) {
+        wslot = ms.wit % BW_SLOTS;
+        ptx::mbar_wait(&C->wfull[wslot], (ms.wit / BW_SLOTS) & 1);
+      }
+      if (c == 0) {
+        if (tid == 0) submark(P, st, 1);
+        ptx::tc_fence_after();
+      }
+      const uint64_t da = da0 + (uint64_t)((as * BA_SLOT_BYTES) >> 4);
+      const uint64_t db = db0 + (uint64_t)((wslot * BW_SLOT_BYTES + j * nt * 128) >> 4);
+      const bool last_in_group = (j == gsz - 1 || c == nk - 1);
+      if (ptx::elect_one()) {
+        ptx::mma_bf16_k64(tmem, da, db, idesc, c > 0 ? 1u : 0u);
+        ptx::mma_commit(&C->aempty[as]);
+        if (last_in_group) ptx::mma_commit(&C->wempty[wslot]);
+        if (c == nk - 1) ptx::mma_commit(&C->accb);
+      }
+      __syncwarp();
+      ++ms.ause;
+      if (last_in_group) ++ms.wit;
+    }
+    if (tid == 0) submark(P, st, 2);    // all MMAs issued
+  }
+
+  // ---- epilogue (all 8 warps: warp w reads TMEM lanes 32*(w%4).., column half w/4)
+  ptx::mbar_wait(&C->accb, ms.accph);
+  ms.accph ^= 1;
+  ptx::tc_fence_after();
+  if (tid == 0) submark(P, st, 3);
+  switch (nt) {
+    case 16: gemm_epilogue<8>(P, st, C, areg, n0, split); break;
+    case 32: gemm_epilogue<16>(P, st, C, areg, n0, split); break;
+    case 64: gemm_epilogue<32>(P, st, C, areg, n0, split); break;
+    default: gemm_epilogue<64>(P, st, C, areg, n0, split); break;
+  }
+  if (tid == 0) submark(P, st, 4);
+}
+
+// ------------------------------------------------------------------ attention stage
+// Attention of head h fused with its slice of the output projection (§6.1 horizontal + §6.2
+// vertical: ctx_h never leaves the SM).  out = ctx Wo^T = sum_h ctx_h Wo[:, h-slice]^T, so CTA
+// (tile j, head h) computes softmax(Q_h K_h^T / sqrt(d)) V_h and multiplies it by the Wo tile
+// [rows j*nt.., cols h*64..] (one 64-wide K chunk, streamed by the weight producer); the result is
+// head h's split-K partial of the out-projection, summed by the LayerNorm row stage.  Every
+// N tile recomputes the (cheap) attention of its head instead of waiting for a grid barrier.
+__device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* wring, char* areg, MmaState& ms) {
+  const int task = blockIdx.x;   // (see the weight producer: task = N tile * heads + head)
+  if (task >= st.ntasks) return;
+  const int h = task % st.heads, jt = task / st.heads;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int S = P.S;
+  char* Qs = areg;                // [128 q][64 d]  one 16 KB atom; later the bf16 ctx_h tile (A operand)
+  char* Ks = areg + 16384;        // [128 keys][64 d]
+  char* Vt = areg + 32768;        // [64 d][128 keys]: 2 atoms of 8 KB (64 keys each)
+  char* Ps = areg + 49152;        // [128 q][128 keys]: 2 atoms of 16 KB
+  const char* tmaps = (const char*)P.tmaps;
+  const uint32_t tmem = C->tmem_base;
+  if (tid == 0) {
+    ptx::mbar_arrive_expect_tx(&C->qkvb, 3 * 16384);
+    ptx::tma_load_3d(Qs, tmaps + 128 * st.qkmap, &C->qkvb, 0, 0, h);
+    ptx::tma_load_3d(Ks, tmaps + 128 * st.qkmap, &C->qkvb, 0, 0, st.heads + h);
+    ptx::tma_load_3d(Vt, tmaps + 128 * st.vtmap, &C->qkvb, 0, 0, h);
+    ptx::tma_load_3d(Vt + 8192, tmaps + 128 * st.vtmap, &C->qkvb, 64, 0, h);
+    submark(P, st, 0);
+  }
+  ptx::mbar_wait(&C->qkvb, ms.qkvph);
+  ms.qkvph ^= 1;
+  if (tid == 0) submark(P, st, 1);
+  // ---- S = Q K^T  (M = 128 queries, N = 128 keys, K = 64) -> TMEM columns [0, 128)
+  if (warp == 0) {
+    ptx::tc_fence_after();
+    const uint32_t idesc = ptx::idesc_bf16(128, 128);
+    const uint64_t dq = ptx::sdesc_sw128(ptx::smem_u32(Qs)), dk = ptx::sdesc_sw128(ptx::smem_u32(Ks));
+    if (ptx::elect_one()) {
+      ptx::mma_bf16_k64(tmem, dq, dk, idesc, 0u);
+      ptx::mma_commit(&C->attb);
+    }
+    __syncwarp();
+  }
+  const int q = warp & 3, half = warp >> 2;
+  const int row = q * 32 + lane;
+  // ---- softmax: warp w owns TMEM lanes 32*(w%4).., the two warps of a lane group split the keys
+  {
+    ptx::mbar_wait(&C->attb, ms.attph);
+    ms.attph ^= 1;
+    ptx::tc_fence_after();
+    if (tid == 0) submark(P, st, 2);
+    const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + half * 64;
+    const float scale = st.scale;
+    float sv[64];
+    ptx::tmem_ld64(tb, sv);
+    float mx = -INFINITY;
+#pragma unroll
+    for (int j = 0; j < 64; ++j) {
+      sv[j] = (half * 64 + j < S) ? sv[j] * scale : -INFINITY;
+      mx = fmaxf(mx, sv[j]);
+    }
+    // each half normalises with its own max; one (max, sum) exchange combines the halves:
+    // z = z_a e^{m_a - m} + z_b e^{m_b - m}, p_j = e^{s_j - m_a} e^{m_a - m} / z
+    float z = 0.f;
+    const float mxs = (mx == -INFINITY) ? 0.f : mx;   // a fully masked half contributes 0
+#pragma unroll
+    for (int j = 0; j < 64; ++j) {
+      sv[j] = __expf(sv[j] - mxs);
+      z += sv[j];
+    }
+    float2* xch = reinterpret_cast<float2*>(Qs);   // [2][128] (max, sum); Q is consumed (S complete)
+    xch[half * 128 + row] = make_float2(mx, z);
+    csync();
+    const float2 o = xch[(half ^ 1) * 128 + row];
+    const float m = fmaxf(mx, o.x);
+    const float zt = z * __expf(mxs - m) + (o.x == -INFINITY ? 0.f : o.y * __expf(o.x - m));
+    const float iz = __expf(mxs - m) / zt;   // p_j = sv[j] * iz
+#pragma unroll
+    for (int c0 = 0; c0 < 64; c0 += 8) {
+      *reinterpret_cast<uint4*>(Ps + half * 16384 + sw128(row, c0 * 2)) =
+          make_uint4(pack_bf16(sv[c0] * iz, sv[c0 + 1] * iz), pack_bf16(sv[c0 + 2] * iz, sv[c0 + 3] * iz),
+                     pack_bf16(sv[c0 + 4] * iz, sv[c0 + 5] * iz), pack_bf16(sv[c0 + 6] * iz, sv[c0 + 7] * iz));
+    }
+    ptx::tc_fence_before();
+  }
+  ptx::fence_proxy_async();
+  csync();
+  if (tid == 0) submark(P, st, 3);
+  // ---- O = P V  (M = 128, N = 64, K = 128 keys) -> TMEM columns [128, 192)
+  if (warp == 0) {
+    ptx::tc_fence_after();
+    const uint32_t idesc = ptx::idesc_bf16(128, 64);
+    const uint64_t dp = ptx::sdesc_sw128(ptx::smem_u32(Ps)), dv = ptx::sdesc_sw128(ptx::smem_u32(Vt));
+    if (ptx::elect_one()) {
+      ptx::mma_bf16_k64(tmem + 128, dp, dv, idesc, 0u);
+      ptx::mma_bf16_k64(tmem + 128, dp + 1024, dv + 512, idesc, 1u);
+      ptx::mma_commit(&C->attb);
+    }
+    __syncwarp();
+  }
+  ptx::mbar_wait(&C->attb, ms.attph);
+  ms.attph ^= 1;
+  ptx::tc_fence_after();
+  if (tid == 0) submark(P, st, 4);
+  // ---- ctx_h (bf16) -> smem as the A operand [128 rows][64 K] of the out-projection tile
+  {
+    float o[32];
+    ptx::tmem_ld32(tmem + 128 + ((uint32_t)(q * 32) << 16) + half * 32, o);
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+      *reinterpret_cast<uint4*>(Qs + sw128(row, (half * 32 + 8 * j) * 2)) =
+          make_uint4(pack_bf16(o[8 * j], o[8 * j + 1]), pack_bf16(o[8 * j + 2], o[8 * j + 3]),
+                     pack_bf16(o[8 * j + 4], o[8 * j + 5]), pack_bf16(o[8 * j + 6], o[8 * j + 7]));
+    ptx::tc_fence_before();
+  }
+  ptx::fence_proxy_async();
+  csync();
+  // ---- partial_h = ctx_h Wo[tile rows, h-slice]^T  (M = 128, N = nt, K = 64) -> TMEM columns [0, nt)
+  if (warp == 0) {
+    const uint32_t wslot = ms.wit % BW_SLOTS;
+    ptx::mbar_wait(&C->wfull[wslot], (ms.wit / BW_SLOTS) & 1);
+    ptx::tc_fence_after();
+    const uint32_t idesc = ptx::idesc_bf16(128, st.nt);
+    const uint64_t da = ptx::sdesc_sw128(ptx::smem_u32(Qs));
+    const uint64_t db = ptx::sdesc_sw128(ptx::smem_u32(wring + wslot * BW_SLOT_BYTES));
+    if (ptx::elect_one()) {
+      ptx::mma_bf16_k64(tmem, da, db, idesc, 0u);
+      ptx::mma_commit(&C->wempty[wslot]);
+      ptx::mma_commit(&C->accb);
+    }
+    __syncwarp();
+    ++ms.wit;
+  }
+  ptx::mbar_wait(&C->accb, ms.accph);
+  ms.accph ^= 1;
+  ptx::tc_fence_after();
+  if (tid == 0) submark(P, st, 5);
+  // split index = head, N tile = jt
+  switch (st.nt) {
+    case 16: gemm_epilogue<8>(P, st, C, areg, jt * st.nt, h); break;
+    case 32: gemm_epilogue<16>(P, st, C, areg, jt * st.nt, h); break;
+    case 64: gemm_epilogue<32>(P, st, C, areg, jt * st.nt, h); break;
+    default: gemm_epilogue<64>(P, st, C, areg, jt * st.nt, h); break;
+  }
+}
+
+// ------------------------------------------------------------------ row stage (one CTA per row)
+__device__ __forceinline__ float block_sum(Ctrl* C, int k, float x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+  if ((threadIdx.x & 31) == 0) C->red[k][threadIdx.x >> 5] = x;
+  csync();
+  float s = 0.f;
+#pragma unroll
+  for (int w = 0; w < 8; ++w) s += C->red[k][w];
+  return s;
+}
+
+constexpr int kRowPer = 3;   // columns per thread: cols <= 768
+constexpr int kMaxSplit = 12;   // split-K partials summed by a LayerNorm row
+__device__ void run_row(const BertParams& P, const BStage& st, Ctrl* C) {
+  const int tid = threadIdx.x;
+  const int S = P.S, cols = st.cols;
+  for (int r = blockIdx.x; r < S; r += gridDim.x) {
+    if (st.row_mode == 0) {
+#pragma unroll
+      for (int i = 0; i < kRowPer; ++i) {
+        const int c = tid + 256 * i;
+        if (c < cols) st.r_out_b[(int64_t)r * cols + c] = bf16_bits(__ldg(st.r_in + (int64_t)r * cols + c));
+      }
+      continue;
+    }
+    // sum of the split-K partials + bias + residual, with gamma / beta: every load of the row is
+    // issued before any is used (one L2 round trip)
+    float v[kRowPer], g[kRowPer], be[kRowPer];
+    float t[kMaxSplit][kRowPer];
+    const int ns = st.r_nsplit;
+    const float* part = st.r_in + (int64_t)r * cols;
+    const int64_t pstride = (int64_t)S * cols;
+#pragma unroll
+    for (int i = 0; i < kRowPer; ++i) {
+      const int c = tid + 256 * i;
+      const bool in = c < cols;
+      v[i] = in ? __ldg(st.r_bias + c) + __ldcg(st.r_res + (int64_t)r * cols + c) : 0.f;
+      g[i] = in ? __ldg(st.r_gamma + c) : 0.f;
+      be[i] = in ? __ldg(st.r_beta + c) : 0.f;
+#pragma unroll
+      for (int u = 0; u < kMaxSplit; ++u) t[u][i] = (u < ns && in) ? __ldcg(part + u * pstride + c) : 0.f;
+    }
+#pragma unroll
+    for (int i = 0; i < kRowPer; ++i) {
+      float a = 0.f;
+#pragma unroll
+      for (int u = 0; u < kMaxSplit; ++u) a += t[u][i];
+      v[i] += a;
+    }
+    if (tid == 0) submark(P, st, 0);
+    float s = 0.f;
+#pragma unroll
+    for (int i = 0; i < kRowPer; ++i) s += v[i];   // out-of-range columns hold 0
+    const float mu = block_sum(C, 0, s) / (float)cols;
+    float q = 0.f;
+#pragma unroll
+    for (int i = 0; i < kRowPer; ++i)
+      if (tid + 256 * i < cols) q += (v[i] - mu) * (v[i] - mu);
+    const float var = block_sum(C, 1, q) / (float)cols;
+    const float rs = rsqrtf(var + st.eps);
+    if (tid == 0) submark(P, st, 1);
+#pragma unroll
+    for (int i = 0; i < kRowPer; ++i) {
+      const int c = tid + 256 * i;
+      if (c < cols) {
+        const float o = (v[i] - mu) * rs * g[i] + be[i];
+        if (st.r_out_f) st.r_out_f[(int64_t)r * cols + c] = o;
+        if (st.r_out_b) st.r_out_b[(int64_t)r * cols + c] = bf16_bits(o);
+      }
+    }
+    csync();   // C->red is reused by the next row of this CTA
+  }
+}
+
+// ------------------------------------------------------------------ the persistent kernel
+__global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_constant__ BertParams P) {
+  extern __shared__ __align__(1024) char smem_raw[];
+  char* smem = (char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  Ctrl* C = reinterpret_cast<Ctrl*>(smem);
+  BStage* sbuf = reinterpret_cast<BStage*>(smem + 1024);   // two staged descriptors
+  char* wring = smem + B_CTRL_BYTES;
+  char* areg = wring + BW_SLOTS * BW_SLOT_BYTES;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  if (tid == 0) {
+    C->cur_stage = -1;
+    for (int i = 0; i < BW_SLOTS; ++i) {
+      ptx::mbar_init(&C->wfull[i], 1);
+      ptx::mbar_init(&C->wempty[i], 1);
+    }
+    for (int i = 0; i < BA_SLOTS; ++i) {
+      ptx::mbar_init(&C->afull[i], 1);
+      ptx::mbar_init(&C->aempty[i], 1);
+    }
+    ptx::mbar_init(&C->accb, 1);
+    ptx::mbar_init(&C->attb, 1);
+    ptx::mbar_init(&C->qkvb, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 0) ptx::tmem_alloc(&C->tmem_base, 256);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+
+  if (warp == 8) {
+    const int lane = tid & 31;
+    if (lane == 0) weight_producer(P, C, wring);   // ---- weight producer
+    if (lane == 1) {
+      // ---- warm L2 with the stage table and every stage's small constant vectors
+      if (blockIdx.x == 0) ptx::prefetch_l2(P.stages, (uint32_t)(P.nstages * sizeof(BStage)));
+      for (int s = blockIdx.x; s < P.nstages; s += gridDim.x) {
+        const BStage* sp = P.stages + s;
+        const int kind = __ldg(&sp->kind);
+        if (kind == BS_ROW && __ldg(&sp->row_mode) == 1) {
+          const uint32_t b = 4u * __ldg(&sp->cols);
+          ptx::prefetch_l2(ldgp(&sp->r_bias), b);
+          ptx::prefetch_l2(ldgp(&sp->r_gamma), b);
+          ptx::prefetch_l2(ldgp(&sp->r_beta), b);
+        } else if (kind == BS_GEMM && __ldg(&sp->epi) != EP_PARTIAL) {
+          ptx::prefetch_l2(ldgp(&sp->bias), 4u * __ldg(&sp->N));
+        }
+      }
+    }
+    return;
+  }
+  // ---- stage executor (warps 0-7).  Stage descriptors are double-buffered in smem: stage s+1's is
+  // fetched while stage s runs, so it is never on the critical path behind a grid barrier.
+  MmaState ms{0u, 0u, 0u, 0u, 0u, 0u};
+  if (tid < (int)(sizeof(BStage) / 16))
+    reinterpret_cast<int4*>(sbuf)[tid] = __ldg(reinterpret_cast<const int4*>(P.stages) + tid);
+  csync();
+  // Barrier participation: only the CTAs with work in stage s arrive at barrier s (its target is
+  // st.workers), and a CTA waits for barrier s-1 only before a stage it works in.  Ordering stays
+  // transitive because every stage has at least one worker, and each worker waited for the
+  // previous barrier before its own arrival.
+  int prev_workers = 0;
+  for (int s = 0; s < P.nstages; ++s) {
+    const BStage& st = sbuf[s & 1];
+    const bool work = has_work(P, st);
+    if (work && s > 0) grid_wait(P, s - 1, prev_workers);
+    prev_workers = st.workers;
+    if (s + 1 < P.nstages && tid < (int)(sizeof(BStage) / 16))
+      reinterpret_cast<int4*>(sbuf + ((s + 1) & 1))[tid] = __ldg(reinterpret_cast<const int4*>(P.stages + s + 1) + tid);
+    if (tid == 0) {
+      mark(P, s);
+      C->cur_stage = s;
+    }
+    if (work) {
+      if (!((P.dbg_skip >> st.kind) & 1)) {
+        switch (st.kind) {
+          case BS_GEMM: run_gemm(P, st, C, wring, areg, ms); break;
+          case BS_ATTN: run_attn(P, st, C, wring, areg, ms); break;
+          default: run_row(P, st, C); break;
+        }
+      } else if ((st.kind == BS_GEMM || st.kind == BS_ATTN) && tid == 0) {
+        // keep the weight ring in step with the producer: consume (and release) this task's groups
+        const int nk = min(st.kchunks, st.K / 64 - (blockIdx.x % st.nsplit) * st.kchunks);
+        const int gsz = wgroup(st.nt);
+        for (int c0 = 0; c0 < nk; c0 += gsz, ++ms.wit) {
+          const uint32_t slot = ms.wit % BW_SLOTS;
+          ptx::mbar_wait(&C->wfull[slot], (ms.wit / BW_SLOTS) & 1);
+          ptx::mbar_arrive(&C->wempty[slot]);
+        }
+      }
+      if (tid == 0) submark(P, st, 6);
+      if (s + 1 < P.nstages) grid_arrive(P, s);
+      if (tid == 0) submark(P, st, 7);
+    }
+    csync();   // descriptor s+1 visible; everyone is done with descriptor s
+  }
+  // ---- exit: the last CTA resets the barrier counters for the next launch
+  csync();
+  if (tid == 0) {
+    __threadfence();
+    const unsigned old = atomicAdd(&P.ctrl[P.nstages], 1u);
+    if (old == gridDim.x - 1) {
+      __threadfence();
+      for (int k = 0; k <= P.nstages; ++k) P.ctrl[k] = 0u;
+    }
+  }
+  if (P.prof && blockIdx.x == 0 && tid == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    P.prof[P.nstages + 1] = t;
+  }
+  ptx::tc_fence_before();
+  csync();
+  if (warp == 0) ptx::tmem_dealloc(C->tmem_base, 256);
+}
+
+}  // namespace bert
+
+cudaError_t bert_launch(const BertParams& prm, int grid, cudaStream_t s) {
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(bert::bert_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, B_SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(BERT_THREADS);
+  cfg.dynamicSmemBytes = B_SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, bert::bert_kernel, prm);
+}
+
+cudaError_t bert_max_active(int* blocks) {
+  cudaError_t e = cudaFuncSetAttribute(bert::bert_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, B_SMEM);
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, bert::bert_kernel, BERT_THREADS, B_SMEM);
+}
+
+}  // namespace souffle

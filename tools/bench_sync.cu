@@ -88,6 +88,84 @@ __global__ void k_grid(unsigned* ctr, long long* out, int rounds) {
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
       }
       __syncthreads();
+    } else if (KIND == 4) {  // hierarchical: group-of-16 counters, last arriver forwards to the root
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence();
+        const unsigned grp = blockIdx.x / 16, gsz = min(16u, gridDim.x - grp * 16);
+        unsigned old = atomicAdd(ctr + 64 + 32 * grp, 1u);
+        if (old + 1 == r * gsz) red_rel(ctr, 1u);
+        const unsigned ngrp = (gridDim.x + 15) / 16;
+        while (ld_acq(ctr) < (unsigned)(r * ngrp)) {}
+      }
+      __syncthreads();
+    } else if (KIND == 5) {  // flag array: each CTA stores its round number; warp 0 polls all flags
+      __syncthreads();
+      unsigned* flags = ctr + 4096;
+      if (threadIdx.x == 0) {
+        __threadfence();
+        asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(flags + blockIdx.x), "r"((unsigned)r) : "memory");
+      }
+      if (threadIdx.x < 32) {
+        while (true) {
+          bool ok = true;
+          for (unsigned c = threadIdx.x; c < gridDim.x; c += 32) ok &= ld_relaxed(flags + c) >= (unsigned)r;
+          if (__all_sync(0xffffffffu, ok)) break;
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      }
+      __syncthreads();
+    } else if (KIND == 6) {  // counter + single poller (CTA 0) + per-CTA release flags
+      __syncthreads();
+      unsigned* flags = ctr + 8192;   // one 128-B line per CTA
+      if (threadIdx.x == 0) {
+        __threadfence();
+        red_rel(ctr, 1u);
+      }
+      if (blockIdx.x == 0) {
+        if (threadIdx.x == 0)
+          while (ld_acq(ctr) < (unsigned)(r * gridDim.x)) {}
+        __syncwarp();
+        if (threadIdx.x < 32)
+          for (unsigned c = threadIdx.x; c < gridDim.x; c += 32)
+            asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flags + 32 * c), "r"((unsigned)r) : "memory");
+      } else if (threadIdx.x == 0) {
+        while (ld_acq(flags + 32 * blockIdx.x) < (unsigned)r) {}
+      }
+      __syncthreads();
+    } else if (KIND == 7) {  // K1 with back-off polling
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        red_rel(ctr, 1u);
+        while (ld_acq(ctr) < (unsigned)(r * gridDim.x)) __nanosleep(100);
+      }
+      __syncthreads();
+    } else if (KIND == 8) {  // 8 counters on separate lines; lanes 0-7 poll all of them
+      __syncthreads();
+      if (threadIdx.x == 0) red_rel(ctr + 32 * (blockIdx.x & 7), 1u);
+      if (threadIdx.x < 32) {
+        const unsigned g = threadIdx.x & 7;
+        const unsigned cnt = gridDim.x / 8 + (g < gridDim.x % 8 ? 1u : 0u);
+        while (true) {
+          bool ok = threadIdx.x >= 8 || ld_relaxed(ctr + 32 * g) >= r * cnt;
+          if (__all_sync(0xffffffffu, ok)) break;
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      }
+      __syncthreads();
+    } else if (KIND == 9) {  // 16 counters on separate lines; lanes 0-15 poll
+      __syncthreads();
+      if (threadIdx.x == 0) red_rel(ctr + 32 * (blockIdx.x & 15), 1u);
+      if (threadIdx.x < 32) {
+        const unsigned g = threadIdx.x & 15;
+        const unsigned cnt = gridDim.x / 16 + (g < gridDim.x % 16 ? 1u : 0u);
+        while (true) {
+          bool ok = threadIdx.x >= 16 || ld_relaxed(ctr + 32 * g) >= r * cnt;
+          if (__all_sync(0xffffffffu, ok)) break;
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      }
+      __syncthreads();
     } else {  // cooperative groups grid.sync()
       cooperative_groups::this_grid().sync();
     }
@@ -119,13 +197,13 @@ int main() {
   for (int i = 0; i < 7; ++i) printf("%-36s %6lld cycles\n", names[i], o[i]);
   int sms;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-  for (int kind = 0; kind < 4; ++kind) {
+  for (int kind = 0; kind < 10; ++kind) {
     for (int grid : {1, 148}) {
-      cudaMemset(buf, 0, 4096);
+      cudaMemset(buf, 0, 1 << 20);
       void* args[] = {&buf, &out, nullptr};
       int rounds = 200;
       args[2] = &rounds;
-      void* fn = kind == 0 ? (void*)k_grid<0> : kind == 1 ? (void*)k_grid<1> : kind == 2 ? (void*)k_grid<2> : (void*)k_grid<3>;
+      void* fn = kind == 0 ? (void*)k_grid<0> : kind == 1 ? (void*)k_grid<1> : kind == 2 ? (void*)k_grid<2> : kind == 3 ? (void*)k_grid<3> : kind == 4 ? (void*)k_grid<4> : kind == 5 ? (void*)k_grid<5> : kind == 6 ? (void*)k_grid<6> : kind == 7 ? (void*)k_grid<7> : kind == 8 ? (void*)k_grid<8> : (void*)k_grid<9>;
       cudaEvent_t a, b;
       cudaEventCreate(&a);
       cudaEventCreate(&b);

@@ -41,8 +41,12 @@ def main():
         s.run()
     torch.cuda.synchronize()
     prof = plan.read_profile(s.ws.data_ptr())
-    kinds = [ln.split()[2] if ln.strip().startswith("||") else ln.split()[1]
-             for ln in plan.describe().splitlines() if ln.startswith("  ")]
+    txt = plan.describe()
+    if txt.startswith("pattern bert:") and "not used" not in txt.splitlines()[0]:
+        kinds = ["CVT"] + ["QKV", "ATTNO", "LN1", "FFN1", "FFN2", "LN2"] * cfg["layers"]
+    else:
+        kinds = [ln.split()[2] if ln.strip().startswith("||") else ln.split()[1]
+                 for ln in txt.splitlines() if ln.startswith("  ")]
     tot = {}
     for i, (k, t) in enumerate(zip(kinds, prof)):
         tot[k] = tot.get(k, 0.0) + t
