@@ -163,6 +163,39 @@ def build_bert(device_index, flags=0):
     return g, plan, sess, X, y, x
 
 
+def build_lstm(device_index, flags=0):
+    import synth
+    from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+    from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+    from paper_conf_asplos_xiazswwyfc24_b200.session import session
+    cfg = synth.LSTM_CFG
+    x = synth.lstm_input(cfg)
+    ps = synth.lstm_params(cfg)
+    g, nm, top, hs, cs = M.lstm(cfg)
+    feed = {nm["X"]: x}
+    for n, p in enumerate(ps):
+        feed[nm[f"W{n}"]], feed[nm[f"U{n}"]] = p["W"], p["U"]
+        feed[nm[f"bih{n}"]], feed[nm[f"bhh{n}"]] = p["b_ih"], p["b_hh"]
+        feed[nm[f"h0_{n}"]] = np.zeros((1, cfg["hidden"]), np.float32)
+        feed[nm[f"c0_{n}"]] = np.zeros((1, cfg["hidden"]), np.float32)
+    plan = g.partition(L.device_query(device_index), flags)
+    return plan, session(g, plan, feed, list(top) + list(hs) + list(cs), device=f"cuda:{device_index}"), cfg
+
+
+def build_mmoe(device_index, flags=0):
+    import synth
+    from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+    from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+    from paper_conf_asplos_xiazswwyfc24_b200.session import session
+    cfg = synth.MMOE_CFG
+    p = synth.mmoe_params(cfg)
+    g, names, outs = M.mmoe(cfg)
+    feed = {names[k]: v for k, v in p.items()}
+    feed[names["x"]] = synth.mmoe_input(cfg)
+    plan = g.partition(L.device_query(device_index), flags)
+    return plan, session(g, plan, feed, outs, device=f"cuda:{device_index}")
+
+
 def time_steps(sess, steps, warmup, flush, stream):
     import torch
     for _ in range(warmup):
@@ -191,6 +224,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-v0", action="store_true")
+    ap.add_argument("--no-models", action="store_true", help="skip the LSTM / MMoE latency extras")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -259,6 +293,25 @@ def main():
         extra["v0_unfused"] = {"latency_us": statistics.median(t0) * 1e3,
                                "launches": plan0.exec_info()["launches"]}
         del sess0, plan0, g0
+    if rank == 0 and not args.no_models:
+        # the other evaluated models of BASELINE.json (latency, same L2-flush protocol)
+        hbm, _, _ = peaks()
+        lplan, lsess, lcfg = build_lstm(local)
+        tl = time_steps(lsess, 20, 3, flush, stream)
+        lw = 2 * 4 * lcfg["hidden"] * (lcfg["input"] + lcfg["hidden"]) * lcfg["layers"]   # bf16 weights, read once
+        lat = statistics.median(tl) * 1e3
+        steps_wf = lcfg["layers"] + lcfg["steps"] - 1
+        extra["lstm"] = {"workload": "LSTM 10 stacked cells, hidden 256, 100 timesteps, batch 1 (bf16 weights, fp32 "
+                                     "activations)", "latency_us": lat, "wavefront_steps": steps_wf,
+                         "us_per_wavefront_step": lat / steps_wf, "weight_bytes": lw,
+                         "hbm_roofline_us": lw / (hbm * 1e3), "kernel": lplan.describe().splitlines()[1][:160]}
+        del lsess, lplan
+        mplan, msess = build_mmoe(local)
+        tm = time_steps(msess, 50, 3, flush, stream)
+        extra["mmoe"] = {"workload": "MMoE 8 experts x 16, 2 tasks, d_in 100, batch 1 (fp32)",
+                         "latency_us": statistics.median(tm) * 1e3, "launches": mplan.exec_info()["launches"],
+                         "stages": mplan.exec_info()["stages"]}
+        del msess, mplan
 
     if rank == 0:
         hbm, tf, src = peaks()

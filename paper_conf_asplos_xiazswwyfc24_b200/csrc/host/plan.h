@@ -6,6 +6,7 @@
 
 #include "../exec_types.h"
 #include "bert.h"
+#include "lstm.h"
 #include "ir.h"
 
 namespace souffle {
@@ -56,6 +57,7 @@ struct Plan {
   bool profiling = false;
   std::vector<uint8_t> host_prog;   // packed program region (uploaded by workspace_init)
   BertPlan bert;                    // pattern lowering (bert.on: kernels/bert.cu runs the program)
+  LstmPlan lstm;                    // pattern lowering (lstm.on: kernels/lstm.cu runs the program)
 };
 
 void lower(Plan& p);              // fills the lowered program + layout (pure host)

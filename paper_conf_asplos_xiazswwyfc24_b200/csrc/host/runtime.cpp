@@ -23,9 +23,12 @@ static int64_t al(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
 souffle_status bert_init(Plan& p, void* ws, void* stream);
 souffle_status bert_run(Plan& p, void* ws, void* stream);
+souffle_status lstm_init(Plan& p, void* ws, void* stream);
+souffle_status lstm_run(Plan& p, void* ws, void* stream);
 
 size_t workspace_bytes(Plan& p) {
   if (p.bert.on) return (size_t)p.bert.total;
+  if (p.lstm.on) return (size_t)p.lstm.total;
   WsLayout& w = p.ws;
   w.ctrl_off = 0;
   // barrier words + stage timestamps + 8 sub-stage marks per stage
@@ -96,6 +99,7 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
   for (size_t s = 0; s < p.buf_ptr.size(); ++s)
     if (!p.buf_ptr[s]) return fail(SOUFFLE_E_STATE, "tensor " + std::to_string(p.buf_node[s]) + " is not bound");
   if (p.bert.on) return bert_init(p, ws, stream);
+  if (p.lstm.on) return lstm_init(p, ws, stream);
   workspace_bytes(p);
   const WsLayout& w = p.ws;
   char* base = (char*)ws;
@@ -155,6 +159,11 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
     std::string why;
     if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
     return bert_run(p, ws, stream);
+  }
+  if (p.lstm.on) {
+    std::string why;
+    if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
+    return lstm_run(p, ws, stream);
   }
   static int max_active = -1;
   if (max_active < 0) {

@@ -1,0 +1,208 @@
+// Persistent wavefront LSTM kernel for sm_100a (§8.4; Fig. 7).
+//
+// One cooperative launch runs the whole stacked LSTM (L layers x T steps).  CTA (l, p) owns hidden
+// units [32p, 32p+32) of layer l: the 128 gate rows (i, f, g, o of those units) of [W_ih | W_hh] are
+// loaded into shared memory ONCE and reused for all T steps (the paper's "weights stay on chip";
+// HBM reads the 10.5 MB of bf16 weights once instead of once per step).  Per step:
+//   wait   point-to-point flags: h(l, t-1) from the NP CTAs of layer l and h(l-1, t) from layer l-1
+//          (release/acquire on per-CTA step counters, no grid barrier; the wavefront is 109 deep)
+//   GEMV   gates = [W_ih | W_hh] [x_t ; h_{t-1}] on CUDA cores, bf16 (or fp32) weights x fp32
+//          activations, fp32 accumulation (activations are never rounded: SURVEY §8(c))
+//   cell   i, f, o = sigmoid, g = tanh; c = f c + i g; h = o tanh(c)  (torch.nn.LSTM semantics)
+//   publish h(l, t) for the 32 units, then the step counter (st.release)
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../lstm_types.h"
+#include "ptx.cuh"
+
+namespace souffle {
+namespace lstm {
+
+__device__ __forceinline__ void st_release(unsigned* p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ float sigm(float x) { return 1.f / (1.f + expf(-x)); }
+
+// 8 consecutive weights of row r (smem) as fp32
+template <bool F32>
+__device__ __forceinline__ void wload8(const char* w, int K, int r, int g, float* o) {
+  if constexpr (F32) {
+    const float4* p = reinterpret_cast<const float4*>(w) + ((int64_t)r * K + 8 * g) / 4;
+    const float4 a = p[0], b = p[1];
+    o[0] = a.x; o[1] = a.y; o[2] = a.z; o[3] = a.w; o[4] = b.x; o[5] = b.y; o[6] = b.z; o[7] = b.w;
+  } else {
+    const uint4 a = *reinterpret_cast<const uint4*>(reinterpret_cast<const uint16_t*>(w) + (int64_t)r * K + 8 * g);
+    const uint32_t u[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      o[2 * j] = __uint_as_float(u[j] << 16);
+      o[2 * j + 1] = __uint_as_float(u[j] & 0xFFFF0000u);
+    }
+  }
+}
+
+template <bool F32>
+__global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_constant__ LstmParams P) {
+  extern __shared__ __align__(16) char smem[];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int l = blockIdx.x / P.NP, p = blockIdx.x % P.NP;
+  const int H = P.H, T = P.T, NP = P.NP, Kst = P.K_max;
+  const LstmLayer& Ly = P.layers[l];
+  const int I = Ly.in_dim, K = I + H;
+  constexpr int ES = F32 ? 4 : 2;
+  char* w = smem;                                                        // [128][Kst] weights
+  float* xh = reinterpret_cast<float*>(smem + (size_t)LSTM_ROWS * Kst * ES);   // [Kst]  [x_t ; h_{t-1}]
+  float* gates = xh + Kst;                                               // [128]
+  float* bias = gates + LSTM_ROWS;                                       // [128] b_ih + b_hh
+
+  // ---- weights of this CTA's 128 gate rows -> shared memory (once for all T steps)
+  {
+    const int vpr = K * ES / 16;   // 16-byte vectors per row
+    for (int e = tid; e < LSTM_ROWS * vpr; e += LSTM_THREADS) {
+      const int r = e / vpr, v = e % vpr;
+      const int grow = (r >> 5) * H + p * LSTM_UNITS + (r & 31);
+      const int col = v * 16 / ES;   // first element of this vector
+      const char* src = col < I ? (const char*)Ly.W + ((int64_t)grow * I + col) * ES
+                                : (const char*)Ly.U + ((int64_t)grow * H + (col - I)) * ES;
+      *reinterpret_cast<uint4*>(w + ((int64_t)r * Kst + col) * ES) = __ldg(reinterpret_cast<const uint4*>(src));
+    }
+    for (int r = tid; r < LSTM_ROWS; r += LSTM_THREADS) {
+      const int grow = (r >> 5) * H + p * LSTM_UNITS + (r & 31);
+      bias[r] = __ldg(Ly.b_ih + grow) + __ldg(Ly.b_hh + grow);
+    }
+  }
+  const int unit = p * LSTM_UNITS + lane;
+  float c = (warp == 0) ? __ldg(Ly.c0 + unit) : 0.f;
+  float h = 0.f;
+  __syncthreads();
+
+  for (int t = 0; t < T; ++t) {
+    // ---- wait for h(l, t-1) (own layer, every part) and h(l-1, t) (previous layer, every part)
+    if (warp == 0) {
+      const unsigned* f = nullptr;
+      unsigned need = 0;
+      if (lane < NP && t > 0) { f = P.flags + l * NP + lane; need = (unsigned)t; }
+      if (lane >= NP && lane < 2 * NP && l > 0) { f = P.flags + (l - 1) * NP + (lane - NP); need = (unsigned)t + 1; }
+      while (true) {
+        const bool ok = f == nullptr || ptx::ld_acquire(f) >= need;
+        if (__all_sync(0xffffffffu, ok)) break;
+      }
+    }
+    __syncthreads();
+    // ---- [x_t ; h_{t-1}] -> shared memory
+    for (int k = tid; k < K; k += LSTM_THREADS) {
+      float v;
+      if (k < I) v = (l == 0) ? __ldg(P.X + (int64_t)t * I + k) : __ldcg(P.hbuf + ((int64_t)(l - 1) * T + t) * H + k);
+      else v = (t == 0) ? __ldg(Ly.h0 + (k - I)) : __ldcg(P.hbuf + ((int64_t)l * T + t - 1) * H + (k - I));
+      xh[k] = v;
+    }
+    __syncthreads();
+    // ---- gates: warp w computes rows 16w..16w+15; lanes split the K columns in groups of 8
+    {
+      float acc[16];
+#pragma unroll
+      for (int i = 0; i < 16; ++i) acc[i] = 0.f;
+      const int ng = K / 8;
+      for (int g = lane; g < ng; g += 32) {
+        const float4 xa = *reinterpret_cast<const float4*>(xh + 8 * g);
+        const float4 xb = *reinterpret_cast<const float4*>(xh + 8 * g + 4);
+        const float xv[8] = {xa.x, xa.y, xa.z, xa.w, xb.x, xb.y, xb.z, xb.w};
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          float wv[8];
+          wload8<F32>(w, Kst, warp * 16 + i, g, wv);
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[i] = fmaf(wv[e], xv[e], acc[i]);
+        }
+      }
+      // transpose-reduce 16 row sums over the 32 lanes (16 shuffles)
+      float v8[8];
+      const bool b4 = lane & 16;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const float send = b4 ? acc[i] : acc[i + 8];
+        const float keep = b4 ? acc[i + 8] : acc[i];
+        v8[i] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
+      }
+      float v4[4];
+      const bool b3 = lane & 8;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float send = b3 ? v8[i] : v8[i + 4];
+        const float keep = b3 ? v8[i + 4] : v8[i];
+        v4[i] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+      }
+      float v2[2];
+      const bool b2 = lane & 4;
+#pragma unroll
+      for (int i = 0; i < 2; ++i) {
+        const float send = b2 ? v4[i] : v4[i + 2];
+        const float keep = b2 ? v4[i + 2] : v4[i];
+        v2[i] = keep + __shfl_xor_sync(0xffffffffu, send, 4);
+      }
+      const bool b1 = lane & 2;
+      float v1 = (b1 ? v2[1] : v2[0]) + __shfl_xor_sync(0xffffffffu, b1 ? v2[0] : v2[1], 2);
+      v1 += __shfl_xor_sync(0xffffffffu, v1, 1);
+      const int r = 8 * ((lane >> 4) & 1) + 4 * ((lane >> 3) & 1) + 2 * ((lane >> 2) & 1) + ((lane >> 1) & 1);
+      if ((lane & 1) == 0) gates[warp * 16 + r] = v1;
+    }
+    __syncthreads();
+    // ---- cell update (warp 0, one unit per lane) and publication of h(l, t)
+    if (warp == 0) {
+      const float gi = gates[lane] + bias[lane];
+      const float gf = gates[32 + lane] + bias[32 + lane];
+      const float gg = gates[64 + lane] + bias[64 + lane];
+      const float go = gates[96 + lane] + bias[96 + lane];
+      c = sigm(gf) * c + sigm(gi) * tanhf(gg);
+      h = sigm(go) * tanhf(c);
+      __stcg(P.hbuf + ((int64_t)l * T + t) * H + unit, h);
+      if (l == P.L - 1) P.top[t][unit] = h;
+      __threadfence();
+      __syncwarp();
+      if (lane == 0) st_release(P.flags + l * NP + p, (unsigned)t + 1);
+    }
+  }
+  if (warp == 0) {
+    Ly.h_n[unit] = h;
+    Ly.c_n[unit] = c;
+  }
+  // ---- exit: the last CTA resets the step counters for the next launch
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();
+    const unsigned old = atomicAdd(P.exit_ctr, 1u);
+    if (old == gridDim.x - 1) {
+      __threadfence();
+      for (int i = 0; i < P.L * P.NP; ++i) P.flags[i] = 0u;
+      *P.exit_ctr = 0u;
+    }
+  }
+}
+
+}  // namespace lstm
+
+size_t lstm_smem_bytes(int K_max, int w_f32) {
+  return (size_t)LSTM_ROWS * K_max * (w_f32 ? 4 : 2) + (size_t)(K_max + 2 * LSTM_ROWS) * 4;
+}
+
+cudaError_t lstm_launch(const LstmParams& prm, int grid, cudaStream_t s) {
+  const size_t smem = lstm_smem_bytes(prm.K_max, prm.w_f32);
+  void (*fn)(LstmParams) = prm.w_f32 ? lstm::lstm_kernel<true> : lstm::lstm_kernel<false>;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(LSTM_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;   // all CTAs co-resident: the flag waits require it
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, fn, prm);
+}
+
+}  // namespace souffle

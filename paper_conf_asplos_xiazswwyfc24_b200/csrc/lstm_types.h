@@ -1,0 +1,42 @@
+// Plain-data structures shared by the host planner (csrc/host/lstm.cpp) and the persistent LSTM
+// kernel (csrc/kernels/lstm.cu).
+//
+// PAPER.md §8.4: a stacked LSTM is one subprogram; Souffle keeps every cell's
+// weights on chip across all time steps and synchronises the wavefront globally instead of
+// relaunching (Table 6: 1911 MB of weight traffic for Rammer vs ~21 MB for Souffle).  Here layer l
+// is owned by NP CTAs; CTA (l, p) keeps the 4*32 gate rows of hidden units [32p, 32p+32) of
+// [W_ih | W_hh] in shared memory for the whole sequence and runs the cells (l, 0..T-1).  The
+// wavefront dependencies (l, t-1) -> (l, t) and (l-1, t) -> (l, t) are point-to-point flags in
+// global memory (release / acquire), not grid barriers.
+#pragma once
+#include <stdint.h>
+
+namespace souffle {
+
+enum { LSTM_THREADS = 256, LSTM_UNITS = 32, LSTM_ROWS = 4 * LSTM_UNITS, LSTM_MAX_SMEM = 200 * 1024 };
+
+struct LstmLayer {
+  const void* W;        // W_ih [4H][I_l] (bf16 or fp32, row-major)
+  const void* U;        // W_hh [4H][H]
+  const float* b_ih;    // [4H]
+  const float* b_hh;    // [4H]
+  const float* h0;      // [H]
+  const float* c0;      // [H]
+  float* h_n;           // [H] final hidden state (output)
+  float* c_n;           // [H] final cell state (output)
+  int32_t in_dim, pad;
+};
+
+struct LstmParams {
+  const LstmLayer* layers;
+  const float* X;        // [T][I_0]
+  float* const* top;     // [T] output pointers: h of the last layer at step t ([H] each)
+  float* hbuf;           // [L][T][H] hidden states (every one written exactly once)
+  unsigned int* flags;   // [L][NP] step counters (t + 1 once h(l, t) of the part is published)
+  unsigned int* exit_ctr;
+  int32_t L, T, H, NP;
+  int32_t w_f32;         // 1: fp32 weights in smem, 0: bf16
+  int32_t K_max;         // max_l (I_l + H): row length of the smem weight tile
+};
+
+}  // namespace souffle

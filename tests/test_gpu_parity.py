@@ -122,8 +122,7 @@ def test_mmoe():
         assert rel_err(r, ref[o]) <= 1e-4
 
 
-def test_lstm_small_fp32():
-    cfg = dict(synth.LSTM_CFG, steps=5, layers=3, hidden=64, input=64, w_dtype="f32")
+def _lstm_case(cfg, flags=0):
     x = synth.lstm_input(cfg)
     ps = synth.lstm_params(cfg)
     spec, names, top, hs, cs = og.lstm(cfg)
@@ -139,7 +138,38 @@ def test_lstm_small_fp32():
 
     ref = te.evaluate(spec, feed_for(names))
     g, gn, gtop, ghs, gcs = M.lstm(cfg)
-    res, plan = run(g, feed_for(gn), gtop)
-    got = np.concatenate(res)
-    want = np.concatenate([ref[t] for t in top])
-    assert rel_err(got, want) <= 1e-4
+    res, plan = run(g, feed_for(gn), list(gtop) + list(ghs) + list(gcs), flags)
+    T = len(gtop)
+    got_top = np.concatenate(res[:T])
+    want_top = np.concatenate([ref[t] for t in top])
+    got_state = np.concatenate(res[T:])
+    want_state = np.concatenate([ref[t] for t in list(hs) + list(cs)])
+    return got_top, want_top, got_state, want_state, plan
+
+
+@pytest.mark.parametrize("flags", [0, L.FLAG_UNFUSED])
+def test_lstm_small_fp32(flags):
+    cfg = dict(synth.LSTM_CFG, steps=5, layers=3, hidden=64, input=64, w_dtype="f32")
+    gt, wt, gs, ws, plan = _lstm_case(cfg, flags)
+    if flags == 0:
+        assert "pattern lstm: 3 layers" in plan.describe()
+    assert rel_err(gt, wt) <= 1e-4
+    assert rel_err(gs, ws) <= 1e-4
+
+
+def test_lstm_ragged_fp32():
+    """3 CTAs per layer, input width != hidden width, odd step count."""
+    cfg = dict(synth.LSTM_CFG, steps=7, layers=2, hidden=96, input=40, w_dtype="f32")
+    gt, wt, gs, ws, plan = _lstm_case(cfg)
+    assert "pattern lstm: 2 layers" in plan.describe()
+    assert rel_err(gt, wt) <= 1e-4
+    assert rel_err(gs, ws) <= 1e-4
+
+
+def test_lstm_full_config_bf16_weights():
+    """BASELINE.json configs[2]: 10 stacked cells, hidden 256, 100 steps, batch 1 (persistent kernel,
+    weights resident on chip).  bf16 weights are exact in the oracle; activations stay fp32."""
+    gt, wt, gs, ws, plan = _lstm_case(synth.LSTM_CFG)
+    assert "pattern lstm: 10 layers x 100 steps" in plan.describe()
+    assert rel_err(gt, wt) <= 1e-4, rel_err(gt, wt)
+    assert rel_err(gs, ws) <= 1e-4
