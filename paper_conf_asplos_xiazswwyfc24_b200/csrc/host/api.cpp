@@ -425,6 +425,12 @@ souffle_status souffle_plan_hgroup(souffle_plan p, souffle_tensor te, int32_t* l
 souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t* stages, int32_t* barriers) {
   return guard([&] {
     Plan& P = PL(p);
+    if (P.mmoe.on) {
+      if (launches) *launches = 1;
+      if (stages) *stages = 5;
+      if (barriers) *barriers = 0;
+      return;
+    }
     if (P.lstm.on) {
       if (launches) *launches = 1;
       if (stages) *stages = P.lstm.L + P.lstm.T - 1;   // wavefront steps

@@ -2,6 +2,7 @@
 // persistent wavefront kernel (kernels/lstm.cu).  PAPER.md §8.4, Table 5 (one
 // kernel), Table 6 (weights read once).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <sstream>
 #include <string>
@@ -130,15 +131,16 @@ void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   lp.NP = lp.H / 32;
   if (2 * lp.NP > 32) return no("more than 16 CTAs per layer");
   lp.K_max = std::max(lp.I, lp.H) + lp.H;
+  if (lp.K_max > 2 * LSTM_THREADS) return no("input + hidden width above 1024");
   const int sms = dev.num_sms > 0 ? dev.num_sms : 148;
   if (lp.L * lp.NP > sms) return no("more CTAs than SMs");
   if (lstm_smem_bytes(lp.K_max, lp.w_f32) > (size_t)LSTM_MAX_SMEM) return no("weights of 32 units do not fit shared memory");
   int64_t o = 0;
-  lp.o_flags = o; o = al(o + 4 * (int64_t)lp.L * lp.NP, 256);
-  lp.o_exit = o; o = al(o + 4, 256);
+  lp.o_gen = o; o = al(o + 8, 256);
   lp.o_layers = o; o = al(o + (int64_t)sizeof(LstmLayer) * lp.L, 256);
   lp.o_top = o; o = al(o + 8 * (int64_t)lp.T, 256);
-  lp.o_hbuf = o; o = al(o + 4 * (int64_t)lp.L * lp.T * lp.H, 256);
+  lp.o_hbuf = o; o = al(o + 8 * (int64_t)lp.L * lp.T * lp.H, 256);
+  lp.o_prof = o; o = al(o + 8 * 4 * (int64_t)lp.T, 256);
   lp.total = al(o, 4096);
   lp.on = true;
 }
@@ -152,7 +154,7 @@ std::string lstm_describe(const LstmPlan& lp) {
   os << "pattern lstm: " << lp.L << " layers x " << lp.T << " steps, H=" << lp.H << " I=" << lp.I << " ("
      << (lp.w_f32 ? "fp32" : "bf16") << " weights) -> 1 persistent launch (kernels/lstm.cu), " << lp.L * lp.NP
      << " CTAs = " << lp.NP << " per layer x 32 units, weights resident in shared memory, wavefront of "
-     << lp.L + lp.T - 1 << " dependent steps synchronised by point-to-point flags\n";
+     << lp.L + lp.T - 1 << " dependent steps synchronised through tagged (value, step) words\n";
   return os.str();
 }
 
@@ -198,15 +200,19 @@ souffle_status lstm_run(Plan& p, void* ws, void* stream) {
   prm.layers = (const LstmLayer*)(base + lp.o_layers);
   prm.X = (const float*)p.buf_ptr[p.node_buf[lp.X]];
   prm.top = (float* const*)(base + lp.o_top);
-  prm.hbuf = (float*)(base + lp.o_hbuf);
-  prm.flags = (unsigned*)(base + lp.o_flags);
-  prm.exit_ctr = (unsigned*)(base + lp.o_exit);
+  prm.hbuf = (uint2*)(base + lp.o_hbuf);
+  prm.gen = (unsigned*)(base + lp.o_gen);
   prm.L = lp.L;
   prm.T = lp.T;
   prm.H = lp.H;
   prm.NP = lp.NP;
   prm.w_f32 = lp.w_f32;
   prm.K_max = lp.K_max;
+  if (p.profiling) {   // debug timeline of one CTA (SOUFFLE_LSTM_PROF_CTA, default the middle layer)
+    prm.prof = (unsigned long long*)(base + lp.o_prof);
+    const char* e = std::getenv("SOUFFLE_LSTM_PROF_CTA");
+    prm.prof_cta = e ? std::atoi(e) : (lp.L / 2) * lp.NP;
+  }
   cudaError_t e = lstm_launch(prm, lp.L * lp.NP, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("lstm launch: ") + cudaGetErrorString(e));
   return SOUFFLE_OK;

@@ -21,7 +21,7 @@ struct LstmPlan {
   std::vector<int> top;                    // [T] output nodes (last layer h at t)
   std::vector<int> hn, cn;                 // [L] final-state output nodes
   // workspace layout
-  int64_t o_flags = 0, o_exit = 0, o_layers = 0, o_top = 0, o_hbuf = 0, total = 0;
+  int64_t o_gen = 0, o_layers = 0, o_top = 0, o_hbuf = 0, o_prof = 0, total = 0;
 };
 
 void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, LstmPlan& lp);

@@ -1,0 +1,177 @@
+// MMoE pattern: strict match of models.mmoe's TE program and launch of the fused kernel
+// (kernels/mmoe.cu).  PAPER.md Table 2, §6.1 (horizontal fusion of the expert and gate GEMMs),
+// Table 5 (one kernel).
+#include <cstring>
+#include <sstream>
+#include <string>
+
+#include <cuda_runtime.h>
+
+#include "../mmoe_types.h"
+#include "plan.h"
+
+namespace souffle {
+
+souffle_status fail(souffle_status c, const std::string& m);
+cudaError_t mmoe_launch(const MmoeParams& prm, cudaStream_t s);
+size_t mmoe_smem_bytes(int B, int D, int E, int De, int T, int Th);
+
+namespace {
+struct Cur {
+  const Graph& g;
+  size_t i = 0;
+  bool ok = true;
+  explicit Cur(const Graph& gr) : g(gr) {}
+  const Node* take(int op) {
+    if (!ok || i >= g.nodes.size() || g.nodes[i].op != op) { ok = false; return nullptr; }
+    return &g.nodes[i++];
+  }
+  int id() const { return (int)i - 1; }
+  int ph(std::vector<int64_t> shape, int dtype) {
+    const Node* n = take(SOUFFLE_OP_PLACEHOLDER);
+    if (!n || !n->is_const || n->shape != shape || n->dtype != dtype) { ok = false; return -1; }
+    return id();
+  }
+  int mm(int a, int b) {
+    const Node* n = take(SOUFFLE_OP_MATMUL);
+    if (!n || n->a != a || n->b != b || !n->trans_b || n->prec != SOUFFLE_F32) { ok = false; return -1; }
+    return id();
+  }
+  int ew(int fn, std::vector<int> in) {
+    const Node* n = take(SOUFFLE_OP_ELEMENTWISE);
+    if (!n || n->fn != fn || n->in != in) { ok = false; return -1; }
+    return id();
+  }
+  int red(int fn, int in) {
+    const Node* n = take(SOUFFLE_OP_REDUCE);
+    if (!n || n->fn != fn || n->in[0] != in || n->axis != 1 || !n->keepdim) { ok = false; return -1; }
+    return id();
+  }
+  int slice(int in, std::vector<int64_t> b, std::vector<int64_t> e) {
+    const Node* n = take(SOUFFLE_OP_SLICE);
+    if (!n || n->in[0] != in || n->begin != b || n->end != e || n->stride != std::vector<int64_t>{1, 1}) {
+      ok = false;
+      return -1;
+    }
+    return id();
+  }
+};
+}  // namespace
+
+void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
+  mp = MmoePlan();
+  auto no = [&](const char* why) { mp.on = false; mp.why_not = why; };
+  if (flags != 0) return no("ablation flags select the generic executor");
+  const auto& N = g.nodes;
+  if (N.size() < 6 || N[0].op != SOUFFLE_OP_PLACEHOLDER || N[0].is_const || N[0].shape.size() != 2 ||
+      N[0].dtype != SOUFFLE_F32 || N[1].op != SOUFFLE_OP_PLACEHOLDER || N[1].shape.size() != 2)
+    return no("not an MMoE program");
+  mp.x = 0;
+  mp.B = (int)N[0].shape[0];
+  mp.D = (int)N[0].shape[1];
+  mp.De = (int)N[1].shape[0];
+  const int wd = N[1].dtype;
+  mp.w_f32 = wd == SOUFFLE_F32;
+  const int64_t B = mp.B, D = mp.D, De = mp.De;
+  Cur c(g);
+  c.i = 1;
+  std::vector<int> ex;
+  // experts: until the first placeholder whose row count differs from De (the first gate)
+  while (c.ok && c.i < N.size() && N[c.i].op == SOUFFLE_OP_PLACEHOLDER && N[c.i].shape.size() == 2 &&
+         N[c.i].shape[0] == De && N[c.i].shape[1] == D) {
+    mp.We.push_back(c.ph({De, D}, wd));
+    int m = c.mm(mp.x, mp.We.back());
+    mp.be.push_back(c.ph({De}, SOUFFLE_F32));
+    ex.push_back(c.ew(SOUFFLE_EW_RELU, {c.ew(SOUFFLE_EW_ADD, {m, mp.be.back()})}));
+  }
+  mp.E = (int)mp.We.size();
+  const int64_t E = mp.E;
+  std::vector<int> gates;
+  while (c.ok && c.i < N.size() && N[c.i].op == SOUFFLE_OP_PLACEHOLDER && N[c.i].shape.size() == 2 &&
+         N[c.i].shape[0] == E && N[c.i].shape[1] == D) {
+    mp.Wg.push_back(c.ph({E, D}, wd));
+    int m = c.mm(mp.x, mp.Wg.back());
+    mp.bg.push_back(c.ph({E}, SOUFFLE_F32));
+    int a = c.ew(SOUFFLE_EW_ADD, {m, mp.bg.back()});
+    int mx = c.red(SOUFFLE_RED_MAX, a);
+    int ee = c.ew(SOUFFLE_EW_EXP, {c.ew(SOUFFLE_EW_SUB, {a, mx})});
+    int z = c.red(SOUFFLE_RED_SUM, ee);
+    gates.push_back(c.ew(SOUFFLE_EW_DIV, {ee, z}));
+  }
+  mp.T = (int)gates.size();
+  if (!c.ok || mp.E < 1 || mp.T < 1) return no("not an MMoE program (experts / gates)");
+  for (int k = 0; k < mp.T && c.ok; ++k) {
+    int acc = -1;
+    for (int e = 0; e < mp.E && c.ok; ++e) {
+      int s = c.slice(gates[k], {0, e}, {B, e + 1});
+      int p = c.ew(SOUFFLE_EW_MUL, {s, ex[e]});
+      acc = acc < 0 ? p : c.ew(SOUFFLE_EW_ADD, {acc, p});
+    }
+    if (!c.ok || c.i >= N.size() || N[c.i].shape.size() != 2) { c.ok = false; break; }
+    if (k == 0) mp.Th = (int)N[c.i].shape[0];
+    const int64_t Th = mp.Th;
+    mp.Wt.push_back(c.ph({Th, De}, wd));
+    int t0 = c.mm(acc, mp.Wt.back());
+    mp.bt.push_back(c.ph({Th}, SOUFFLE_F32));
+    int t2 = c.ew(SOUFFLE_EW_RELU, {c.ew(SOUFFLE_EW_ADD, {t0, mp.bt.back()})});
+    mp.Wo.push_back(c.ph({1, Th}, wd));
+    int y0 = c.mm(t2, mp.Wo.back());
+    mp.bo.push_back(c.ph({1}, SOUFFLE_F32));
+    mp.y.push_back(c.ew(SOUFFLE_EW_ADD, {y0, mp.bo.back()}));
+  }
+  if (!c.ok || c.i != N.size()) return no("not an MMoE program (towers)");
+  if (g.outputs != mp.y) return no("outputs are not the task towers");
+  if (mp.E > MMOE_MAX_E || mp.T > MMOE_MAX_T || mp.B > MMOE_MAX_B) return no("too many experts / tasks / rows");
+  const int epv = mp.w_f32 ? 4 : 8;   // weight tensors are staged by bulk copies of 16-byte multiples
+  if ((int64_t)mp.De * mp.D % epv || (int64_t)mp.E * mp.D % epv || (int64_t)mp.Th * mp.De % epv || mp.Th % epv)
+    return no("weight tensor sizes must be multiples of 16 bytes");
+  if (mmoe_smem_bytes(mp.B, mp.D, mp.E, mp.De, mp.T, mp.Th) > (size_t)MMOE_MAX_SMEM)
+    return no("parameters do not fit one CTA's shared memory");
+  mp.on = true;
+}
+
+std::string mmoe_describe(const MmoePlan& mp) {
+  std::ostringstream os;
+  if (!mp.on) {
+    os << "pattern mmoe: not used (" << mp.why_not << ")\n";
+    return os.str();
+  }
+  os << "pattern mmoe: " << mp.E << " experts x " << mp.De << ", " << mp.T << " tasks, d_in " << mp.D << ", batch "
+     << mp.B << " -> 1 launch (kernels/mmoe.cu): horizontally fused expert+gate GEMM, softmax gates, mixture and "
+        "towers in one CTA, parameters staged once in shared memory\n";
+  return os.str();
+}
+
+souffle_status mmoe_run(Plan& p, void* ws, void* stream) {
+  (void)ws;
+  MmoePlan& mp = p.mmoe;
+  auto ptr = [&](int node) -> void* { return p.buf_ptr[p.node_buf[node]]; };
+  MmoeParams prm;
+  std::memset(&prm, 0, sizeof(prm));
+  prm.x = (const float*)ptr(mp.x);
+  for (int e = 0; e < mp.E; ++e) {
+    prm.We[e] = ptr(mp.We[e]);
+    prm.be[e] = (const float*)ptr(mp.be[e]);
+  }
+  for (int k = 0; k < mp.T; ++k) {
+    prm.Wg[k] = ptr(mp.Wg[k]);
+    prm.bg[k] = (const float*)ptr(mp.bg[k]);
+    prm.Wt[k] = ptr(mp.Wt[k]);
+    prm.bt[k] = (const float*)ptr(mp.bt[k]);
+    prm.Wo[k] = ptr(mp.Wo[k]);
+    prm.bo[k] = (const float*)ptr(mp.bo[k]);
+    prm.y[k] = (float*)ptr(mp.y[k]);
+  }
+  prm.B = mp.B; prm.D = mp.D; prm.E = mp.E; prm.De = mp.De; prm.T = mp.T; prm.Th = mp.Th;
+  prm.w_f32 = mp.w_f32;
+  for (int k = 0; k < mp.E; ++k)
+    if ((uintptr_t)prm.We[k] & 15) return fail(SOUFFLE_E_INVALID_ARG, "MMoE weights must be 16-byte aligned");
+  for (int k = 0; k < mp.T; ++k)
+    if (((uintptr_t)prm.Wg[k] | (uintptr_t)prm.Wt[k] | (uintptr_t)prm.Wo[k]) & 15)
+      return fail(SOUFFLE_E_INVALID_ARG, "MMoE weights must be 16-byte aligned");
+  cudaError_t e = mmoe_launch(prm, (cudaStream_t)stream);
+  if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("mmoe launch: ") + cudaGetErrorString(e));
+  return SOUFFLE_OK;
+}
+
+}  // namespace souffle

@@ -1,0 +1,24 @@
+// Pattern lowering for multi-gate mixture-of-experts (Table 2): when the whole TE
+// program is the MMoE built by models.mmoe (experts Linear+ReLU, per-task softmax gates, gated sum,
+// towers Linear+ReLU -> Linear), it runs on the single-CTA fused kernel in kernels/mmoe.cu.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "ir.h"
+
+namespace souffle {
+
+struct MmoePlan {
+  bool on = false;
+  std::string why_not;
+  int B = 0, D = 0, E = 0, De = 0, T = 0, Th = 0, w_f32 = 0;
+  int x = -1;
+  std::vector<int> We, be, Wg, bg, Wt, bt, Wo, bo, y;
+};
+
+void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp);
+std::string mmoe_describe(const MmoePlan& mp);
+
+}  // namespace souffle

@@ -7,6 +7,7 @@
 #include "../exec_types.h"
 #include "bert.h"
 #include "lstm.h"
+#include "mmoe.h"
 #include "ir.h"
 
 namespace souffle {
@@ -58,6 +59,7 @@ struct Plan {
   std::vector<uint8_t> host_prog;   // packed program region (uploaded by workspace_init)
   BertPlan bert;                    // pattern lowering (bert.on: kernels/bert.cu runs the program)
   LstmPlan lstm;                    // pattern lowering (lstm.on: kernels/lstm.cu runs the program)
+  MmoePlan mmoe;                    // pattern lowering (mmoe.on: kernels/mmoe.cu runs the program)
 };
 
 void lower(Plan& p);              // fills the lowered program + layout (pure host)

@@ -25,10 +25,12 @@ souffle_status bert_init(Plan& p, void* ws, void* stream);
 souffle_status bert_run(Plan& p, void* ws, void* stream);
 souffle_status lstm_init(Plan& p, void* ws, void* stream);
 souffle_status lstm_run(Plan& p, void* ws, void* stream);
+souffle_status mmoe_run(Plan& p, void* ws, void* stream);
 
 size_t workspace_bytes(Plan& p) {
   if (p.bert.on) return (size_t)p.bert.total;
   if (p.lstm.on) return (size_t)p.lstm.total;
+  if (p.mmoe.on) return 256;
   WsLayout& w = p.ws;
   w.ctrl_off = 0;
   // barrier words + stage timestamps + 8 sub-stage marks per stage
@@ -100,6 +102,11 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
     if (!p.buf_ptr[s]) return fail(SOUFFLE_E_STATE, "tensor " + std::to_string(p.buf_node[s]) + " is not bound");
   if (p.bert.on) return bert_init(p, ws, stream);
   if (p.lstm.on) return lstm_init(p, ws, stream);
+  if (p.mmoe.on) {
+    p.inited_ws = ws;
+    p.dirty = false;
+    return SOUFFLE_OK;
+  }
   workspace_bytes(p);
   const WsLayout& w = p.ws;
   char* base = (char*)ws;
@@ -165,6 +172,11 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
     if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
     return lstm_run(p, ws, stream);
   }
+  if (p.mmoe.on) {
+    std::string why;
+    if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
+    return mmoe_run(p, ws, stream);
+  }
   static int max_active = -1;
   if (max_active < 0) {
     std::string why;
@@ -214,6 +226,15 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
 }
 
 souffle_status read_profile_raw(Plan& p, void* ws, unsigned long long* out, int cap, int* n) {
+  if (p.lstm.on) {   // [T][4] timestamps of the profiled CTA: step start, operands in smem, gates, -
+    const size_t cnt = 4 * (size_t)p.lstm.T;
+    if ((size_t)cap < cnt) return fail(SOUFFLE_E_INVALID_ARG, "profile buffer too small");
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e == cudaSuccess) e = cudaMemcpy(out, (char*)ws + p.lstm.o_prof, cnt * 8, cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("profile read: ") + cudaGetErrorString(e));
+    *n = (int)cnt;
+    return SOUFFLE_OK;
+  }
   if (p.bert.on) {   // [0, ns): stage starts, ns+1: end; then 16 sub-stage marks per stage
     const size_t cnt = 17 * (size_t)p.bert.nstages + 2;
     if ((size_t)cap < cnt) return fail(SOUFFLE_E_INVALID_ARG, "profile buffer too small");

@@ -4,12 +4,13 @@
 // units [32p, 32p+32) of layer l: the 128 gate rows (i, f, g, o of those units) of [W_ih | W_hh] are
 // loaded into shared memory ONCE and reused for all T steps (the paper's "weights stay on chip";
 // HBM reads the 10.5 MB of bf16 weights once instead of once per step).  Per step:
-//   wait   point-to-point flags: h(l, t-1) from the NP CTAs of layer l and h(l-1, t) from layer l-1
-//          (release/acquire on per-CTA step counters, no grid barrier; the wavefront is 109 deep)
+//   wait   h(l, t-1) and h(l-1, t) are read as (value, tag) words straight from L2, spinning until
+//          every tag carries this run's step (one round trip = readiness + data; no grid barrier,
+//          no fence; the wavefront is L + T - 1 = 109 cells deep)
 //   GEMV   gates = [W_ih | W_hh] [x_t ; h_{t-1}] on CUDA cores, bf16 (or fp32) weights x fp32
 //          activations, fp32 accumulation (activations are never rounded: SURVEY §8(c))
 //   cell   i, f, o = sigmoid, g = tanh; c = f c + i g; h = o tanh(c)  (torch.nn.LSTM semantics)
-//   publish h(l, t) for the 32 units, then the step counter (st.release)
+//   publish h(l, t) for the 32 units as (value, tag) 64-bit words
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -20,9 +21,6 @@
 namespace souffle {
 namespace lstm {
 
-__device__ __forceinline__ void st_release(unsigned* p, unsigned v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
 __device__ __forceinline__ float sigm(float x) { return 1.f / (1.f + expf(-x)); }
 
 // 8 consecutive weights of row r (smem) as fp32
@@ -78,77 +76,96 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
   float h = 0.f;
   __syncthreads();
 
+  auto stamp = [&](int t, int k) {
+    if (P.prof && blockIdx.x == P.prof_cta && tid == 0) {
+      unsigned long long g;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+      P.prof[4 * t + k] = g;
+    }
+  };
+  const unsigned gen = *(volatile unsigned*)P.gen;   // written by the previous launch's last CTA
+  const unsigned tag0 = gen * (unsigned)(T + 1) + 1u;
   for (int t = 0; t < T; ++t) {
-    // ---- wait for h(l, t-1) (own layer, every part) and h(l-1, t) (previous layer, every part)
-    if (warp == 0) {
-      const unsigned* f = nullptr;
-      unsigned need = 0;
-      if (lane < NP && t > 0) { f = P.flags + l * NP + lane; need = (unsigned)t; }
-      if (lane >= NP && lane < 2 * NP && l > 0) { f = P.flags + (l - 1) * NP + (lane - NP); need = (unsigned)t + 1; }
-      while (true) {
-        const bool ok = f == nullptr || ptx::ld_acquire(f) >= need;
-        if (__all_sync(0xffffffffu, ok)) break;
+    stamp(t, 0);
+    // ---- [x_t ; h_{t-1}] -> shared memory; operands produced by other CTAs are spun on until their
+    // tag is this run's step (x of layer l > 0 is h(l-1, t); h is h(l, t-1))
+    {
+      // every operand word of this thread is requested before any is waited on (one round trip)
+      constexpr int kMaxPer = 2;   // K <= 2 * LSTM_THREADS
+      const uint2* src[kMaxPer];
+      unsigned want[kMaxPer];
+      unsigned long long w64[kMaxPer];
+#pragma unroll
+      for (int i = 0; i < kMaxPer; ++i) {
+        const int k = tid + i * LSTM_THREADS;
+        src[i] = nullptr;
+        if (k >= K) continue;
+        if (k < I && l == 0) {
+          xh[k] = __ldg(P.X + (int64_t)t * I + k);
+        } else if (k >= I && t == 0) {
+          xh[k] = __ldg(Ly.h0 + (k - I));
+        } else {
+          src[i] = (k < I) ? P.hbuf + ((int64_t)(l - 1) * T + t) * H + k : P.hbuf + ((int64_t)l * T + t - 1) * H + (k - I);
+          want[i] = tag0 + (unsigned)(k < I ? t : t - 1);
+          asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w64[i]) : "l"(src[i]) : "memory");
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < kMaxPer; ++i) {
+        if (src[i] == nullptr) continue;
+        while ((unsigned)(w64[i] >> 32) != want[i])   // one single-copy-atomic word: tag in the high half
+          asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w64[i]) : "l"(src[i]) : "memory");
+        xh[tid + i * LSTM_THREADS] = __uint_as_float((unsigned)w64[i]);
       }
     }
     __syncthreads();
-    // ---- [x_t ; h_{t-1}] -> shared memory
-    for (int k = tid; k < K; k += LSTM_THREADS) {
-      float v;
-      if (k < I) v = (l == 0) ? __ldg(P.X + (int64_t)t * I + k) : __ldcg(P.hbuf + ((int64_t)(l - 1) * T + t) * H + k);
-      else v = (t == 0) ? __ldg(Ly.h0 + (k - I)) : __ldcg(P.hbuf + ((int64_t)l * T + t - 1) * H + (k - I));
-      xh[k] = v;
-    }
-    __syncthreads();
-    // ---- gates: warp w computes rows 16w..16w+15; lanes split the K columns in groups of 8
+    stamp(t, 1);
+    // ---- gates: warp w computes rows RPW*w ..; lanes split the K columns in groups of 8
     {
-      float acc[16];
+      constexpr int RPW = LSTM_ROWS / (LSTM_THREADS / 32);   // rows per warp (8 with 16 warps)
+      static_assert(RPW == 8, "reduction below assumes 8 rows per warp");
+      float acc[RPW];
 #pragma unroll
-      for (int i = 0; i < 16; ++i) acc[i] = 0.f;
+      for (int i = 0; i < RPW; ++i) acc[i] = 0.f;
       const int ng = K / 8;
       for (int g = lane; g < ng; g += 32) {
         const float4 xa = *reinterpret_cast<const float4*>(xh + 8 * g);
         const float4 xb = *reinterpret_cast<const float4*>(xh + 8 * g + 4);
         const float xv[8] = {xa.x, xa.y, xa.z, xa.w, xb.x, xb.y, xb.z, xb.w};
+        float wv[RPW][8];
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          float wv[8];
-          wload8<F32>(w, Kst, warp * 16 + i, g, wv);
+        for (int i = 0; i < RPW; ++i) wload8<F32>(w, Kst, warp * RPW + i, g, wv[i]);
 #pragma unroll
-          for (int e = 0; e < 8; ++e) acc[i] = fmaf(wv[e], xv[e], acc[i]);
-        }
+        for (int i = 0; i < RPW; ++i)
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[i] = fmaf(wv[i][e], xv[e], acc[i]);
       }
-      // transpose-reduce 16 row sums over the 32 lanes (16 shuffles)
-      float v8[8];
+      // transpose-reduce 8 row sums over the 32 lanes (4 + 2 + 1 + 2 shuffles)
+      float v4[4];
       const bool b4 = lane & 16;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const float send = b4 ? acc[i] : acc[i + 8];
-        const float keep = b4 ? acc[i + 8] : acc[i];
-        v8[i] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
-      }
-      float v4[4];
-      const bool b3 = lane & 8;
-#pragma unroll
       for (int i = 0; i < 4; ++i) {
-        const float send = b3 ? v8[i] : v8[i + 4];
-        const float keep = b3 ? v8[i + 4] : v8[i];
-        v4[i] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+        const float send = b4 ? acc[i] : acc[i + 4];
+        const float keep = b4 ? acc[i + 4] : acc[i];
+        v4[i] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
       }
       float v2[2];
-      const bool b2 = lane & 4;
+      const bool b3 = lane & 8;
 #pragma unroll
       for (int i = 0; i < 2; ++i) {
-        const float send = b2 ? v4[i] : v4[i + 2];
-        const float keep = b2 ? v4[i + 2] : v4[i];
-        v2[i] = keep + __shfl_xor_sync(0xffffffffu, send, 4);
+        const float send = b3 ? v4[i] : v4[i + 2];
+        const float keep = b3 ? v4[i + 2] : v4[i];
+        v2[i] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
       }
-      const bool b1 = lane & 2;
-      float v1 = (b1 ? v2[1] : v2[0]) + __shfl_xor_sync(0xffffffffu, b1 ? v2[0] : v2[1], 2);
+      const bool b2 = lane & 4;
+      float v1 = (b2 ? v2[1] : v2[0]) + __shfl_xor_sync(0xffffffffu, b2 ? v2[0] : v2[1], 4);
+      v1 += __shfl_xor_sync(0xffffffffu, v1, 2);
       v1 += __shfl_xor_sync(0xffffffffu, v1, 1);
-      const int r = 8 * ((lane >> 4) & 1) + 4 * ((lane >> 3) & 1) + 2 * ((lane >> 2) & 1) + ((lane >> 1) & 1);
-      if ((lane & 1) == 0) gates[warp * 16 + r] = v1;
+      const int r = 4 * ((lane >> 4) & 1) + 2 * ((lane >> 3) & 1) + ((lane >> 2) & 1);
+      if ((lane & 3) == 0) gates[warp * RPW + r] = v1;
     }
     __syncthreads();
+    stamp(t, 2);
     // ---- cell update (warp 0, one unit per lane) and publication of h(l, t)
     if (warp == 0) {
       const float gi = gates[lane] + bias[lane];
@@ -157,26 +174,25 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
       const float go = gates[96 + lane] + bias[96 + lane];
       c = sigm(gf) * c + sigm(gi) * tanhf(gg);
       h = sigm(go) * tanhf(c);
-      __stcg(P.hbuf + ((int64_t)l * T + t) * H + unit, h);
       if (l == P.L - 1) P.top[t][unit] = h;
-      __threadfence();
-      __syncwarp();
-      if (lane == 0) st_release(P.flags + l * NP + p, (unsigned)t + 1);
+      const unsigned long long w64 = ((unsigned long long)(tag0 + (unsigned)t) << 32) | __float_as_uint(h);
+      uint2* dst = P.hbuf + ((int64_t)l * T + t) * H + unit;
+      asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(dst), "l"(w64) : "memory");
     }
   }
   if (warp == 0) {
     Ly.h_n[unit] = h;
     Ly.c_n[unit] = c;
   }
-  // ---- exit: the last CTA resets the step counters for the next launch
+  // ---- exit: the last CTA advances the run generation (tags of the next launch differ)
   __syncthreads();
   if (tid == 0) {
     __threadfence();
-    const unsigned old = atomicAdd(P.exit_ctr, 1u);
+    const unsigned old = atomicAdd(P.gen + 1, 1u);
     if (old == gridDim.x - 1) {
+      P.gen[1] = 0u;
+      P.gen[0] = gen + 1u;
       __threadfence();
-      for (int i = 0; i < P.L * P.NP; ++i) P.flags[i] = 0u;
-      *P.exit_ctr = 0u;
     }
   }
 }

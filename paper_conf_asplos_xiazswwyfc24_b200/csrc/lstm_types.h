@@ -6,14 +6,16 @@
 // relaunching (Table 6: 1911 MB of weight traffic for Rammer vs ~21 MB for Souffle).  Here layer l
 // is owned by NP CTAs; CTA (l, p) keeps the 4*32 gate rows of hidden units [32p, 32p+32) of
 // [W_ih | W_hh] in shared memory for the whole sequence and runs the cells (l, 0..T-1).  The
-// wavefront dependencies (l, t-1) -> (l, t) and (l-1, t) -> (l, t) are point-to-point flags in
-// global memory (release / acquire), not grid barriers.
+// wavefront dependencies (l, t-1) -> (l, t) and (l-1, t) -> (l, t) are carried by the data itself:
+// every published h value is a 64-bit word (fp32 value, 32-bit tag = step of this run), so a
+// consumer's single L2 round trip both detects readiness and fetches the operand (no fence, no
+// separate flag; the "LL" low-latency protocol idea), and no grid barrier is involved.
 #pragma once
 #include <stdint.h>
 
 namespace souffle {
 
-enum { LSTM_THREADS = 256, LSTM_UNITS = 32, LSTM_ROWS = 4 * LSTM_UNITS, LSTM_MAX_SMEM = 200 * 1024 };
+enum { LSTM_THREADS = 512, LSTM_UNITS = 32, LSTM_ROWS = 4 * LSTM_UNITS, LSTM_MAX_SMEM = 200 * 1024 };
 
 struct LstmLayer {
   const void* W;        // W_ih [4H][I_l] (bf16 or fp32, row-major)
@@ -31,12 +33,13 @@ struct LstmParams {
   const LstmLayer* layers;
   const float* X;        // [T][I_0]
   float* const* top;     // [T] output pointers: h of the last layer at step t ([H] each)
-  float* hbuf;           // [L][T][H] hidden states (every one written exactly once)
-  unsigned int* flags;   // [L][NP] step counters (t + 1 once h(l, t) of the part is published)
-  unsigned int* exit_ctr;
+  uint2* hbuf;           // [L][T][H] (value bits, tag) of every hidden state, written exactly once per run
+  unsigned int* gen;     // [0]: run generation (tags of this run are gen * (T + 1) + t + 1); [1]: exit counter
   int32_t L, T, H, NP;
   int32_t w_f32;         // 1: fp32 weights in smem, 0: bf16
   int32_t K_max;         // max_l (I_l + H): row length of the smem weight tile
+  unsigned long long* prof;   // debug: per-step timestamps of CTA prof_cta ([T][4]), null if off
+  int32_t prof_cta, pad;
 };
 
 }  // namespace souffle

@@ -1,0 +1,26 @@
+// Plain-data structures shared by the host planner (csrc/host/mmoe.cpp) and the fused MMoE kernel
+// (csrc/kernels/mmoe.cu).  PAPER.md Table 2 L1308 (MMoE), §6.1 horizontal transformation (the 8
+// expert GEMMs and the 2 gate GEMMs share x and run as one fused GEMM), Table 5 (one kernel).
+#pragma once
+#include <stdint.h>
+
+namespace souffle {
+
+enum { MMOE_THREADS = 256, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
+
+struct MmoeParams {
+  const float* x;                  // [B][D]
+  const void* We[MMOE_MAX_E];      // expert weights [De][D]
+  const float* be[MMOE_MAX_E];     // [De]
+  const void* Wg[MMOE_MAX_T];      // gate weights [E][D]
+  const float* bg[MMOE_MAX_T];     // [E]
+  const void* Wt[MMOE_MAX_T];      // tower hidden [Th][De]
+  const float* bt[MMOE_MAX_T];     // [Th]
+  const void* Wo[MMOE_MAX_T];      // tower output [1][Th]
+  const float* bo[MMOE_MAX_T];     // [1]
+  float* y[MMOE_MAX_T];            // outputs [B][1]
+  int32_t B, D, E, De, T, Th;
+  int32_t w_f32, pad;
+};
+
+}  // namespace souffle

@@ -106,8 +106,12 @@ def test_bert_base_bf16(layers, flags):
         assert float(np.abs(out - exact).max()) <= 2e-2
 
 
-def test_mmoe():
-    cfg = synth.MMOE_CFG
+@pytest.mark.parametrize("cfg,flags", [
+    (synth.MMOE_CFG, 0),
+    (synth.MMOE_CFG, L.FLAG_UNFUSED),
+    (dict(synth.MMOE_CFG, batch=4, experts=5, tasks=3, expert_dim=24, tower_hidden=16, d_in=72, w_dtype="bf16"), 0),
+])
+def test_mmoe(cfg, flags):
     p = synth.mmoe_params(cfg)
     x = synth.mmoe_input(cfg)
     spec, names, outs = og.mmoe(cfg)
@@ -117,12 +121,14 @@ def test_mmoe():
     g, gn, gouts = M.mmoe(cfg)
     gfeed = {gn[k]: v for k, v in p.items()}
     gfeed[gn["x"]] = x
-    res, plan = run(g, gfeed, gouts)
+    res, plan = run(g, gfeed, gouts, flags)
+    if flags == 0:
+        assert "pattern mmoe:" in plan.describe() and "not used" not in plan.describe().splitlines()[2]
     for o, r in zip(outs, res):
         assert rel_err(r, ref[o]) <= 1e-4
 
 
-def _lstm_case(cfg, flags=0):
+def _lstm_case(cfg, flags=0, reps=1):
     x = synth.lstm_input(cfg)
     ps = synth.lstm_params(cfg)
     spec, names, top, hs, cs = og.lstm(cfg)
@@ -138,7 +144,12 @@ def _lstm_case(cfg, flags=0):
 
     ref = te.evaluate(spec, feed_for(names))
     g, gn, gtop, ghs, gcs = M.lstm(cfg)
-    res, plan = run(g, feed_for(gn), list(gtop) + list(ghs) + list(gcs), flags)
+    outs = list(gtop) + list(ghs) + list(gcs)
+    plan = g.partition(L.device_query(0), flags)
+    s = session(g, plan, feed_for(gn), outs)
+    for _ in range(reps):   # repeated launches reuse the workspace (run-generation tags)
+        s.run()
+    res = [s.result(o) for o in outs]
     T = len(gtop)
     got_top = np.concatenate(res[:T])
     want_top = np.concatenate([ref[t] for t in top])
@@ -169,7 +180,7 @@ def test_lstm_ragged_fp32():
 def test_lstm_full_config_bf16_weights():
     """BASELINE.json configs[2]: 10 stacked cells, hidden 256, 100 steps, batch 1 (persistent kernel,
     weights resident on chip).  bf16 weights are exact in the oracle; activations stay fp32."""
-    gt, wt, gs, ws, plan = _lstm_case(synth.LSTM_CFG)
+    gt, wt, gs, ws, plan = _lstm_case(synth.LSTM_CFG, reps=3)
     assert "pattern lstm: 10 layers x 100 steps" in plan.describe()
     assert rel_err(gt, wt) <= 1e-4, rel_err(gt, wt)
     assert rel_err(gs, ws) <= 1e-4

@@ -1,1 +1,1 @@
-timeout 300 python bench.py --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/b7.log 2>&1; echo rc=$? >> gpurun_out/b7.log
+timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/p9.log 2>&1; echo rc=$? >> gpurun_out/p9.log
