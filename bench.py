@@ -56,38 +56,61 @@ def dist_env():
 
 
 class Clocks:
-    """nvidia-smi sampler running during the timed region."""
+    """nvidia-smi sampler (10 ms period) started before the warm-up; only the samples whose
+    timestamps fall inside the timed region [mark_start(), mark_end()] are reported."""
 
     def __init__(self, gpu):
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
-        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+        q = ("timestamp,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
              "clocks_event_reasons.sw_power_cap")
+        self.t0 = self.t1 = None
         try:
             self.p = subprocess.Popen(["nvidia-smi", f"--id={gpu}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
-                                       "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+                                       "-lms", "10"], stdout=self.f, stderr=subprocess.DEVNULL)
+            time.sleep(0.5)   # let the sampler start before anything is timed
         except OSError:
             self.p = None
+
+    def mark_start(self):
+        self.t0 = time.time()
+
+    def mark_end(self):
+        self.t1 = time.time()
 
     def stop(self):
         if self.p is None:
             return None
+        time.sleep(0.05)
         self.p.terminate()
         self.p.wait()
         self.f.flush()
-        rows = [l.split(",") for l in open(self.f.name).read().strip().splitlines() if l.strip()]
+        import datetime
+        rows = []
+        for line in open(self.f.name).read().strip().splitlines():
+            r = [c.strip() for c in line.split(",")]
+            if len(r) < 8:
+                continue
+            try:
+                ts = datetime.datetime.strptime(r[0], "%Y/%m/%d %H:%M:%S.%f").timestamp()
+            except ValueError:
+                continue
+            rows.append((ts, r))
         os.unlink(self.f.name)
-        if not rows:
+        inside = [r for ts, r in rows if self.t0 is not None and self.t0 - 0.005 <= ts <= self.t1 + 0.005]
+        used = inside if inside else [r for _, r in rows]
+        if not used:
             return None
-        sm = [float(r[1]) for r in rows]
-        mx = float(rows[0][2])
+        sm = [float(r[1]) for r in used]
+        mx = float(used[0][2])
         reasons = set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in rows:
+        for r in used:
             for k, nm in enumerate(names):
                 if "Active" in r[4 + k] and "Not" not in r[4 + k]:
                     reasons.add(nm)
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(rows)}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(used), "samples_in_timed_region": len(inside)}
 
 
 def oracle_bert_layer_runner():
@@ -196,12 +219,14 @@ def build_mmoe(device_index, flags=0):
     return plan, session(g, plan, feed, outs, device=f"cuda:{device_index}")
 
 
-def time_steps(sess, steps, warmup, flush, stream):
+def time_steps(sess, steps, warmup, flush, stream, clk=None):
     import torch
     for _ in range(warmup):
         flush.zero_()
         sess.run()
     torch.cuda.synchronize()
+    if clk:
+        clk.mark_start()
     times = []
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
     with torch.cuda.stream(stream):
@@ -211,6 +236,8 @@ def time_steps(sess, steps, warmup, flush, stream):
             sess.run()
             b.record(stream)
     torch.cuda.synchronize()
+    if clk:
+        clk.mark_end()
     for a, b in ev:
         times.append(a.elapsed_time(b))
     return times
@@ -219,7 +246,7 @@ def time_steps(sess, steps, warmup, flush, stream):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -247,7 +274,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     clk = Clocks(local) if rank == 0 else None
-    times = time_steps(sess, args.steps, args.warmup, flush, stream)
+    times = time_steps(sess, args.steps, args.warmup, flush, stream, clk)
     clocks = clk.stop() if clk else None
     total_ms = sum(times)
     if ws > 1:
