@@ -20,7 +20,7 @@ from collections import deque
 
 from .te import infer_shapes
 
-OR_OPS = {"ew", "reshape", "permute", "slice"}
+OR_OPS = {"ew", "reshape", "permute", "slice", "roll"}
 MR_OPS = {"matmul", "reduce"}
 
 
@@ -210,6 +210,8 @@ def or_map(n, shapes, i, j_pos, idx):
         return src
     if op == "slice":
         return [b + v * s for b, v, s in zip(n["begin"], idx, n["stride"])]
+    if op == "roll":   # quasi-affine: (i - shift) mod n
+        return [(v - sh) % d for v, sh, d in zip(idx, n["shifts"], shapes[i])]
     raise ValueError(op)
 
 

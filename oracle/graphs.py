@@ -277,3 +277,136 @@ def lstm(cfg):
         b.out(h[n])
         b.out(c[n])
     return b.spec(), names, top, list(h), list(c)
+
+
+# ---------------------------------------------------------------- Swin-Transformer (Table 2)
+def _swin_res(cfg, i):
+    return cfg["image"] // cfg["patch"] // (2 ** i)
+
+
+def _swin_shift(cfg, i, j):
+    w = cfg["window"]
+    return 0 if (j % 2 == 0 or w >= _swin_res(cfg, i)) else w // 2
+
+
+def _swin_ln(b, x, C, eps, names, gk, bk):
+    out, (g, be) = _layernorm(b, x, C, eps, gk, bk)
+    names[gk], names[bk] = g, be
+    return out
+
+
+def swin_block(b, x, cfg, B, R, C, nh, shift, gb, names):
+    """One Swin block (pre-LN; W-MSA / SW-MSA then MLP), torchvision `SwinTransformerBlock`:
+    x = x + proj(window_attention(LN1(x))); x = x + W2 gelu(W1 LN2(x)).  x is [B*R*R, C] (b, h, w
+    row-major).  Cyclic shift = roll TE; window partition / reverse = reshape + permute TEs."""
+    w = cfg["window"]
+    n = R // w
+    nW = n * n
+    d = C // nh
+    prec = cfg["gemm_dtype"]
+    pre = f"b{gb}."
+    h = _swin_ln(b, x, C, cfg["eps"], names, pre + "g1", pre + "be1")
+    t = b.reshape(h, (B, R, R, C))
+    if shift:
+        t = b._add({"op": "roll", "in": t, "shifts": [0, -shift, -shift, 0]})
+    t = b.reshape(t, (B, n, w, n, w, C))
+    t = b.permute(t, (0, 1, 3, 2, 4, 5))
+    t = b.reshape(t, (B * nW * w * w, C))
+    Wqkv = b.ph((3 * C, C), dtype=prec)
+    qkv = b.mm(t, Wqkv, 1, prec)
+    bqkv = b.ph((3 * C,))
+    qkv = b.ew("add", qkv, bqkv)
+    names[pre + "Wqkv"], names[pre + "bqkv"] = Wqkv, bqkv
+    qkv = b.reshape(qkv, (B * nW, w * w, 3, nh, d))
+    qkv = b.permute(qkv, (2, 0, 3, 1, 4))
+    qs, ks, vs = [b.reshape(b.slice(qkv, (k, 0, 0, 0, 0), (k + 1, B * nW, nh, w * w, d), (1, 1, 1, 1, 1)),
+                            (B * nW, nh, w * w, d)) for k in range(3)]
+    qs = b.ew("mul_scalar", qs, scalar=float(d) ** -0.5)
+    a = b.mm(qs, ks, 1, prec)
+    bias = b.ph((nh, w * w, w * w))
+    names[pre + "bias"] = bias
+    a = b.ew("add", a, bias)
+    if shift:
+        a = b.reshape(a, (B, nW, nh, w * w, w * w))
+        mask = b.ph((nW, 1, w * w, w * w))
+        names[pre + "mask"] = mask
+        a = b.ew("add", a, mask)
+        a = b.reshape(a, (B * nW, nh, w * w, w * w))
+    mx = b.red("max", a, 3)
+    e = b.ew("exp", b.ew("sub", a, mx))
+    z = b.red("sum", e, 3)
+    p = b.ew("div", e, z)
+    o = b.mm(p, vs, 0, prec)
+    o = b.reshape(b.permute(o, (0, 2, 1, 3)), (B * nW * w * w, C))
+    Wp = b.ph((C, C), dtype=prec)
+    o = b.mm(o, Wp, 1, prec)
+    bp = b.ph((C,))
+    o = b.ew("add", o, bp)
+    names[pre + "Wproj"], names[pre + "bproj"] = Wp, bp
+    o = b.reshape(o, (B, n, n, w, w, C))
+    o = b.permute(o, (0, 1, 3, 2, 4, 5))
+    o = b.reshape(o, (B, R, R, C))
+    if shift:
+        o = b._add({"op": "roll", "in": o, "shifts": [0, shift, shift, 0]})
+    o = b.reshape(o, (B * R * R, C))
+    x = b.ew("add", x, o)
+    h = _swin_ln(b, x, C, cfg["eps"], names, pre + "g2", pre + "be2")
+    F = cfg["mlp_ratio"] * C
+    W1 = b.ph((F, C), dtype=prec)
+    f = b.mm(h, W1, 1, prec)
+    b1 = b.ph((F,))
+    f = b.ew("gelu_erf", b.ew("add", f, b1))
+    W2 = b.ph((C, F), dtype=prec)
+    f = b.mm(f, W2, 1, prec)
+    b2 = b.ph((C,))
+    f = b.ew("add", f, b2)
+    names.update({pre + "W1": W1, pre + "b1": b1, pre + "W2": W2, pre + "b2": b2})
+    return b.ew("add", x, f)
+
+
+def swin(cfg):
+    """Swin-Transformer (torchvision `SwinTransformer` v1 semantics) as a TE program.
+    Returns (spec, names: placeholder name -> id, image id, logits id)."""
+    b = SpecBuilder()
+    names = {}
+    B, p, C = cfg["batch"], cfg["patch"], cfg["embed"]
+    prec = cfg["gemm_dtype"]
+    img = cfg["image"]
+    R = img // p
+    x = b.ph((B, 3, img, img), const=0)
+    # patch embedding: Conv2d(3, C, p, stride p) == im2col (reshape + permute) + GEMM
+    t = b.reshape(x, (B, 3, R, p, R, p))
+    t = b.permute(t, (0, 2, 4, 1, 3, 5))
+    t = b.reshape(t, (B * R * R, 3 * p * p))
+    Wpe = b.ph((C, 3 * p * p), dtype=prec)
+    t = b.mm(t, Wpe, 1, prec)
+    bpe = b.ph((C,))
+    t = b.ew("add", t, bpe)
+    names["Wpe"], names["bpe"] = Wpe, bpe
+    h = _swin_ln(b, t, C, cfg["eps"], names, "gpe", "bepe")
+    gb = 0
+    for i, (depth, nh) in enumerate(zip(cfg["depths"], cfg["heads"])):
+        R = _swin_res(cfg, i)
+        for j in range(depth):
+            h = swin_block(b, h, cfg, B, R, C, nh, _swin_shift(cfg, i, j), gb, names)
+            gb += 1
+        if i < len(cfg["depths"]) - 1:
+            # patch merging: cat(x[0::2,0::2], x[1::2,0::2], x[0::2,1::2], x[1::2,1::2]) -> LN -> Linear
+            t = b.reshape(h, (B, R // 2, 2, R // 2, 2, C))
+            t = b.permute(t, (0, 1, 3, 4, 2, 5))
+            t = b.reshape(t, (B * (R // 2) ** 2, 4 * C))
+            t = _swin_ln(b, t, 4 * C, cfg["eps"], names, f"m{i}.g", f"m{i}.be")
+            Wm = b.ph((2 * C, 4 * C), dtype=prec)
+            h = b.mm(t, Wm, 1, prec)
+            names[f"m{i}.W"] = Wm
+            C *= 2
+    R = _swin_res(cfg, len(cfg["depths"]) - 1)
+    h = _swin_ln(b, h, C, cfg["eps"], names, "gn", "ben")
+    h = b.red("mean", b.reshape(h, (B, R * R, C)), 1, keepdim=0)
+    Wh = b.ph((cfg["classes"], C), dtype=prec)
+    y = b.mm(h, Wh, 1, prec)
+    bh = b.ph((cfg["classes"],))
+    y = b.ew("add", y, bh)
+    names["Wh"], names["bh"] = Wh, bh
+    b.out(y)
+    return b.spec(), names, x, y

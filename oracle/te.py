@@ -17,6 +17,9 @@ Per-op semantics (the readings are listed in DESIGN.md "Readings of the paper"):
   ew(fn, inputs, scalar): numpy broadcasting over trailing dims.
   reduce(fn, axis, keepdim): sum / max / mean over ONE axis.
   reshape / permute / strided slice: pure index maps (one-relies-on-one, §5.2).
+  roll(shifts): cyclic shift, out[..., i, ...] = in[..., (i - shift) mod n, ...] per dim
+        (torch.roll / np.roll semantics) -- a quasi-affine (mod) index map (§5.2
+        "quasi-affine maps"); Swin-Transformer's shifted windows (Table 2).
 
 Two evaluation modes: vectorised numpy (default) and `brute=True`, which evaluates every output
 element by its definition in pure Python loops (tiny shapes only) and pins the vectorised mode.
@@ -85,6 +88,9 @@ def infer_shapes(spec):
             shp = tuple(s[p] for p in n["perm"])
         elif op == "slice":
             shp = tuple(slice_len(b, e, st) for b, e, st in zip(n["begin"], n["end"], n["stride"]))
+        elif op == "roll":
+            shp = tuple(shapes[n["in"]])
+            assert len(n["shifts"]) == len(shp)
         else:
             raise ValueError(op)
         shapes.append(shp)
@@ -223,6 +229,8 @@ def _vec(n, vals, bf16_operands):
     if op == "slice":
         sl = tuple(slice(b, e, s) for b, e, s in zip(n["begin"], n["end"], n["stride"]))
         return vals[n["in"]][sl]
+    if op == "roll":
+        return np.roll(vals[n["in"]], tuple(n["shifts"]), axis=tuple(range(len(n["shifts"]))))
     raise ValueError(op)
 
 
@@ -300,6 +308,9 @@ def _brute(n, vals, shapes, i, bf16_operands):
             out[idx] = vals[n["in"]][tuple(src)]
         elif op == "slice":
             src = tuple(b + v * s for b, v, s in zip(n["begin"], idx, n["stride"]))
+            out[idx] = vals[n["in"]][src]
+        elif op == "roll":
+            src = tuple((v - sh) % d for v, sh, d in zip(idx, n["shifts"], shp))
             out[idx] = vals[n["in"]][src]
         else:
             raise ValueError(op)
