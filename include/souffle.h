@@ -59,7 +59,8 @@ enum { SOUFFLE_F32 = 0, SOUFFLE_BF16 = 1 };
 
 /* node kinds reported by souffle_graph_node */
 enum { SOUFFLE_OP_PLACEHOLDER = 0, SOUFFLE_OP_MATMUL = 1, SOUFFLE_OP_ELEMENTWISE = 2,
-       SOUFFLE_OP_REDUCE = 3, SOUFFLE_OP_RESHAPE = 4, SOUFFLE_OP_PERMUTE = 5, SOUFFLE_OP_SLICE = 6 };
+       SOUFFLE_OP_REDUCE = 3, SOUFFLE_OP_RESHAPE = 4, SOUFFLE_OP_PERMUTE = 5, SOUFFLE_OP_SLICE = 6,
+       SOUFFLE_OP_ROLL = 7 };
 
 /* elementwise functions (one-relies-on-one TEs, §5.2).  Binary ops use numpy
  * broadcasting over trailing dims; *_SCALAR ops take the `scalar` argument. */
@@ -100,6 +101,11 @@ souffle_status souffle_permute(souffle_graph g, souffle_tensor in, const int32_t
 /* strided slice, half-open [begin, end) with positive stride per dim (Fig. 4) */
 souffle_status souffle_slice(souffle_graph g, souffle_tensor in, const int64_t* begin, const int64_t* end,
                              const int64_t* stride, souffle_tensor* out);
+/* cyclic shift (torch.roll / np.roll): out[.., i_d, ..] = in[.., (i_d - shifts[d]) mod n_d, ..] for every
+ * dim d (shifts has ndim entries, any sign).  A one-relies-on-one TE whose index map is quasi-affine
+ * (mod by a constant, §5.2 P:L897-898 "quasi-affine maps"): Swin-Transformer's shifted windows
+ * (Table 2).  Errors: E_INVALID_ARG on a null argument. */
+souffle_status souffle_roll(souffle_graph g, souffle_tensor in, const int64_t* shifts, souffle_tensor* out);
 souffle_status souffle_mark_output(souffle_graph g, souffle_tensor t);
 
 /* graph introspection (used by tests to compare with the oracle's own builders) */

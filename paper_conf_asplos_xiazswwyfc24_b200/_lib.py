@@ -9,7 +9,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libsouffle.so")
 
 F32, BF16 = 0, 1
-OP_PLACEHOLDER, OP_MATMUL, OP_ELEMENTWISE, OP_REDUCE, OP_RESHAPE, OP_PERMUTE, OP_SLICE = range(7)
+OP_PLACEHOLDER, OP_MATMUL, OP_ELEMENTWISE, OP_REDUCE, OP_RESHAPE, OP_PERMUTE, OP_SLICE, OP_ROLL = range(8)
 EW = dict(add=0, sub=1, mul=2, div=3, max=4, exp=5, tanh=6, sigmoid=7, relu=8, gelu_erf=9, rsqrt=10, neg=11,
           add_scalar=12, mul_scalar=13)
 RED = dict(sum=0, max=1, mean=2)
@@ -42,6 +42,7 @@ _SIGS = {
     "souffle_reduce": [C.c_void_p, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32)],
     "souffle_reshape": [C.c_void_p, C.c_int32, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32)],
     "souffle_permute": [C.c_void_p, C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_int32)],
+    "souffle_roll": [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32)],
     "souffle_slice": [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int64), C.POINTER(C.c_int64),
                       C.POINTER(C.c_int32)],
     "souffle_mark_output": [C.c_void_p, C.c_int32],
@@ -157,6 +158,9 @@ class Graph:
 
     def slice(self, x, begin, end, stride):
         return self._out(self.lib.souffle_slice, x, _i64(begin), _i64(end), _i64(stride))
+
+    def roll(self, x, shifts):
+        return self._out(self.lib.souffle_roll, x, _i64(shifts))
 
     def mark_output(self, t):
         check(self.lib.souffle_mark_output(self.h, t))

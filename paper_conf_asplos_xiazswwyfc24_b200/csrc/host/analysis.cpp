@@ -39,7 +39,7 @@ std::vector<int> distinct_inputs(const Node& n) {
 
 bool is_or_op(int op) {
   return op == SOUFFLE_OP_ELEMENTWISE || op == SOUFFLE_OP_RESHAPE || op == SOUFFLE_OP_PERMUTE ||
-         op == SOUFFLE_OP_SLICE;
+         op == SOUFFLE_OP_SLICE || op == SOUFFLE_OP_ROLL;
 }
 bool is_mr_op(int op) { return op == SOUFFLE_OP_MATMUL || op == SOUFFLE_OP_REDUCE; }
 
@@ -260,6 +260,12 @@ void or_map(const Graph& g, int node, int pos, const int64_t* idx, int64_t* out)
       break;
     case SOUFFLE_OP_SLICE:
       for (int d = 0; d < nd; ++d) out[d] = n.begin[d] + idx[d] * n.stride[d];
+      break;
+    case SOUFFLE_OP_ROLL:   // quasi-affine: (i - shift) mod n
+      for (int d = 0; d < nd; ++d) {
+        const int64_t m = n.shape[d];
+        out[d] = ((idx[d] - n.shifts[d]) % m + m) % m;
+      }
       break;
     default: throw std::runtime_error("or_map on a non-OR TE");
   }

@@ -252,6 +252,21 @@ souffle_status souffle_slice(souffle_graph g, souffle_tensor in, const int64_t* 
   });
 }
 
+souffle_status souffle_roll(souffle_graph g, souffle_tensor in, const int64_t* shifts, souffle_tensor* out) {
+  return guard([&] {
+    Graph& gr = G(g);
+    check_t(gr, in);
+    need(out && shifts, SOUFFLE_E_INVALID_ARG, "null argument");
+    const auto& s = gr.nodes[in].shape;
+    Node n;
+    n.op = SOUFFLE_OP_ROLL;
+    n.in = {in};
+    n.shape = s;
+    for (size_t d = 0; d < s.size(); ++d) n.shifts.push_back(((shifts[d] % s[d]) + s[d]) % s[d]);
+    *out = push(gr, n);
+  });
+}
+
 souffle_status souffle_mark_output(souffle_graph g, souffle_tensor t) {
   return guard([&] {
     Graph& gr = G(g);

@@ -25,6 +25,8 @@ struct Node {
   // permute / slice
   std::vector<int> perm;
   std::vector<int64_t> begin, end, stride;
+  // roll
+  std::vector<int64_t> shifts;
   // partition resource override (§5.4 "Get required resource")
   bool res_override = false;
   int64_t r_grid = 0, r_smem = 0;

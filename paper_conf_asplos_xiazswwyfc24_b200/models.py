@@ -203,3 +203,120 @@ def from_spec(spec):
     for o in spec["outputs"]:
         g.mark_output(o)
     return g
+
+
+# ---------------------------------------------------------------- Swin-Transformer (Table 2)
+def _swin_res(cfg, i):
+    return cfg["image"] // cfg["patch"] // (2 ** i)
+
+
+def _swin_shift(cfg, i, j):
+    """Odd blocks use shifted windows (w // 2) unless the window already covers the whole map."""
+    w = cfg["window"]
+    return 0 if (j % 2 == 0 or w >= _swin_res(cfg, i)) else w // 2
+
+
+def _swin_block(g, x, cfg, B, R, C, nh, shift, gb, names):
+    """x [B*R*R, C] -> x + proj(W-MSA / SW-MSA(LN1 x)) -> + MLP(LN2 x).  The cyclic shift is a roll
+    TE and the window partition / reverse are reshape + permute TEs: all one-relies-on-one index
+    maps that the lowering folds into the neighbouring GEMM loads and stores (§6.2)."""
+    w = cfg["window"]
+    n = R // w
+    nW, L2 = n * n, w * w
+    d = C // nh
+    prec = _DT[cfg["gemm_dtype"]]
+    pre = f"b{gb}."
+    h = _layernorm(g, x, C, cfg["eps"], names, pre + "g1", pre + "be1")
+    t = g.reshape(h, (B, R, R, C))
+    if shift:
+        t = g.roll(t, (0, -shift, -shift, 0))
+    t = g.reshape(g.permute(g.reshape(t, (B, n, w, n, w, C)), (0, 1, 3, 2, 4, 5)), (B * nW * L2, C))
+    Wqkv = g.placeholder((3 * C, C), prec)
+    qkv = g.matmul(t, Wqkv, True, prec)
+    bqkv = g.placeholder((3 * C,))
+    qkv = g.ew("add", qkv, bqkv)
+    names[pre + "Wqkv"], names[pre + "bqkv"] = Wqkv, bqkv
+    qkv = g.permute(g.reshape(qkv, (B * nW, L2, 3, nh, d)), (2, 0, 3, 1, 4))
+    q, k, v = [g.reshape(g.slice(qkv, (j, 0, 0, 0, 0), (j + 1, B * nW, nh, L2, d), (1, 1, 1, 1, 1)), (B * nW, nh, L2, d))
+               for j in range(3)]
+    q = g.ew("mul_scalar", q, scalar=float(d) ** -0.5)
+    a = g.matmul(q, k, True, prec)
+    bias = g.placeholder((nh, L2, L2))
+    names[pre + "bias"] = bias
+    a = g.ew("add", a, bias)
+    if shift:
+        a = g.reshape(a, (B, nW, nh, L2, L2))
+        mask = g.placeholder((nW, 1, L2, L2))
+        names[pre + "mask"] = mask
+        a = g.reshape(g.ew("add", a, mask), (B * nW, nh, L2, L2))
+    mx = g.reduce("max", a, 3)
+    e = g.ew("exp", g.ew("sub", a, mx))
+    z = g.reduce("sum", e, 3)
+    p = g.ew("div", e, z)
+    o = g.matmul(p, v, False, prec)
+    o = g.reshape(g.permute(o, (0, 2, 1, 3)), (B * nW * L2, C))
+    Wp = g.placeholder((C, C), prec)
+    o = g.matmul(o, Wp, True, prec)
+    bp = g.placeholder((C,))
+    o = g.ew("add", o, bp)
+    names[pre + "Wproj"], names[pre + "bproj"] = Wp, bp
+    o = g.reshape(g.permute(g.reshape(o, (B, n, n, w, w, C)), (0, 1, 3, 2, 4, 5)), (B, R, R, C))
+    if shift:
+        o = g.roll(o, (0, shift, shift, 0))
+    x = g.ew("add", x, g.reshape(o, (B * R * R, C)))
+    h = _layernorm(g, x, C, cfg["eps"], names, pre + "g2", pre + "be2")
+    F = cfg["mlp_ratio"] * C
+    W1 = g.placeholder((F, C), prec)
+    f = g.matmul(h, W1, True, prec)
+    b1 = g.placeholder((F,))
+    f = g.ew("gelu_erf", g.ew("add", f, b1))
+    W2 = g.placeholder((C, F), prec)
+    f = g.matmul(f, W2, True, prec)
+    b2 = g.placeholder((C,))
+    f = g.ew("add", f, b2)
+    names.update({pre + "W1": W1, pre + "b1": b1, pre + "W2": W2, pre + "b2": b2})
+    return g.ew("add", x, f)
+
+
+def swin(cfg):
+    """Swin-Transformer (torchvision SwinTransformer v1 semantics).  Returns (graph, names, image id,
+    logits id); `names` maps every other placeholder to the key used by synth.swin.swin_feed_values."""
+    g = L.Graph()
+    names = {}
+    B, p, C, img = cfg["batch"], cfg["patch"], cfg["embed"], cfg["image"]
+    prec = _DT[cfg["gemm_dtype"]]
+    R = img // p
+    x = g.placeholder((B, 3, img, img), L.F32, const=False)
+    # patch embedding: Conv2d(3, C, p, stride p) = im2col (reshape + permute) + GEMM
+    t = g.reshape(g.permute(g.reshape(x, (B, 3, R, p, R, p)), (0, 2, 4, 1, 3, 5)), (B * R * R, 3 * p * p))
+    Wpe = g.placeholder((C, 3 * p * p), prec)
+    t = g.matmul(t, Wpe, True, prec)
+    bpe = g.placeholder((C,))
+    t = g.ew("add", t, bpe)
+    names["Wpe"], names["bpe"] = Wpe, bpe
+    h = _layernorm(g, t, C, cfg["eps"], names, "gpe", "bepe")
+    gb = 0
+    for i, (depth, nh) in enumerate(zip(cfg["depths"], cfg["heads"])):
+        R = _swin_res(cfg, i)
+        for j in range(depth):
+            h = _swin_block(g, h, cfg, B, R, C, nh, _swin_shift(cfg, i, j), gb, names)
+            gb += 1
+        if i < len(cfg["depths"]) - 1:
+            # patch merging: channel blocks (h even, w even), (odd, even), (even, odd), (odd, odd)
+            t = g.reshape(g.permute(g.reshape(h, (B, R // 2, 2, R // 2, 2, C)), (0, 1, 3, 4, 2, 5)),
+                          (B * (R // 2) ** 2, 4 * C))
+            t = _layernorm(g, t, 4 * C, cfg["eps"], names, f"m{i}.g", f"m{i}.be")
+            Wm = g.placeholder((2 * C, 4 * C), prec)
+            h = g.matmul(t, Wm, True, prec)
+            names[f"m{i}.W"] = Wm
+            C *= 2
+    R = _swin_res(cfg, len(cfg["depths"]) - 1)
+    h = _layernorm(g, h, C, cfg["eps"], names, "gn", "ben")
+    h = g.reduce("mean", g.reshape(h, (B, R * R, C)), 1, False)
+    Wh = g.placeholder((cfg["classes"], C), prec)
+    y = g.matmul(h, Wh, True, prec)
+    bh = g.placeholder((cfg["classes"],))
+    y = g.ew("add", y, bh)
+    names["Wh"], names["bh"] = Wh, bh
+    g.mark_output(y)
+    return g, names, x, y

@@ -172,3 +172,26 @@ def test_bert_base_lowering_structure():
     v0 = g.partition(L.device_b200(), flags=L.FLAG_UNFUSED).exec_info()
     te_count = plan.num_tes()
     assert v0["launches"] == te_count                 # V0: one kernel per TE (Fig. 5(a))
+
+
+def test_swin_graph_matches_oracle_builder_and_analysis():
+    import synth.swin as S
+    cfg = S.SWIN_TINY
+    spec, names, x, y = og.swin(cfg)
+    g, gnames, gx, gy = M.swin(cfg)
+    assert g.num_nodes() == len(spec["nodes"]) and gnames == names and (gx, gy) == (x, y)
+    shapes = te.infer_shapes(spec)
+    opmap = {"placeholder": 0, "matmul": 1, "ew": 2, "reduce": 3, "reshape": 4, "permute": 5, "slice": 6, "roll": 7}
+    for i, nd in enumerate(spec["nodes"]):
+        op, shp, dt = g.node(i)
+        assert op == opmap[nd["op"]] and shp == shapes[i], i
+    dev = L.device_b200()
+    plan = g.partition(dev)
+    _check_plan_vs_oracle(spec, plan, dev, check_maps=False)
+    # index maps through the roll / window-partition chains, bit-exact with the oracle
+    for t, nd in enumerate(spec["nodes"]):
+        if nd["op"] == "roll":
+            for s in (nd["in"], t - 3):
+                ref = an.index_map(spec, t, s)
+                if ref is not None:
+                    assert plan.index_map(t, s, int(np.prod(shapes[t]))) == ref, (t, s)

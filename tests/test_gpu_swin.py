@@ -1,0 +1,61 @@
+"""GPU parity for Swin-Transformer (Table 2) on the generic
+fused-subprogram executor (the roll / window-partition index maps are folded into the GEMM loads
+and stores, §6.2).  Tolerances as in test_gpu_parity.py: fp32 path rel 1e-4; bf16-operand path
+max abs 2e-2 against the oracle's bf16-operand emulation."""
+import numpy as np
+import pytest
+
+import synth.swin as S
+from oracle import graphs as og
+from oracle import te
+from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+from paper_conf_asplos_xiazswwyfc24_b200.session import session
+
+pytestmark = pytest.mark.gpu
+
+
+def rel_err(g, o):
+    rms = np.sqrt(np.mean(o * o)) + 1e-30
+    return float(np.max(np.abs(g - o) / np.maximum(np.abs(o), rms)))
+
+
+def _run(cfg, flags=0, bf16=False):
+    P = S.swin_params(cfg)
+    fv = S.swin_feed_values(cfg, P)
+    img = S.swin_input(cfg)
+    g, names, x, y = M.swin(cfg)
+    feed = {names[k]: v for k, v in fv.items()}
+    feed[x] = img
+    plan = g.partition(L.device_query(0), flags)
+    s = session(g, plan, feed, [y])
+    s.run()
+    got = s.result(y)
+    s.run()                                   # a second launch reuses the workspace
+    again = s.result(y)
+    spec, onames, ox, oy = og.swin(cfg)
+    ref = te.evaluate(spec, feed, bf16_operands=bf16)[oy]
+    return got, again, ref, plan
+
+
+@pytest.mark.parametrize("batch", [1, 2])
+@pytest.mark.parametrize("flags", [0, L.FLAG_UNFUSED])
+def test_swin_tiny_fp32(batch, flags):
+    got, again, ref, plan = _run(dict(S.SWIN_TINY, batch=batch), flags)
+    assert rel_err(got, ref) <= 1e-4, plan.describe()[:2000]
+    assert rel_err(again, ref) <= 1e-4
+
+
+def test_swin_tiny_bf16_tensor_cores():
+    """embed 64 so every Linear has K % 64 == 0 and runs on the tcgen05 GEMM stage."""
+    cfg = dict(S.SWIN_TINY, embed=64, heads=(2, 4), gemm_dtype="bf16")
+    got, again, ref, plan = _run(cfg, bf16=True)
+    assert "GEMM_TC" in plan.describe()
+    assert np.max(np.abs(got - ref)) <= 2e-2
+    assert np.max(np.abs(again - ref)) <= 2e-2
+
+
+def test_swin_b_batch1_full_size():
+    got, again, ref, plan = _run(S.SWIN_B, bf16=True)
+    assert got.shape == (1, 1000)
+    assert np.max(np.abs(got - ref)) <= 2e-2, np.max(np.abs(got - ref))
