@@ -219,6 +219,23 @@ def build_mmoe(device_index, flags=0):
     return plan, session(g, plan, feed, outs, device=f"cuda:{device_index}")
 
 
+def build_swin(device_index, batch=1, flags=0):
+    import synth.swin as S
+    from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+    from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+    from paper_conf_asplos_xiazswwyfc24_b200.session import session
+    cfg = dict(S.SWIN_B, batch=batch)
+    fv = S.swin_feed_values(cfg, S.swin_params(cfg))
+    g, names, x, y = M.swin(cfg)
+    feed = {names[k]: v for k, v in fv.items()}
+    feed[x] = S.swin_input(cfg)
+    plan = g.partition(L.device_query(device_index), flags)
+    return plan, session(g, plan, feed, [y], device=f"cuda:{device_index}"), cfg
+
+
+SWIN_FLOPS = 30.86e9   # per 224x224 image (torch flop counter)
+
+
 def time_steps(sess, steps, warmup, flush, stream, clk=None):
     import torch
     for _ in range(warmup):
@@ -339,6 +356,17 @@ def main():
                          "latency_us": statistics.median(tm) * 1e3, "launches": mplan.exec_info()["launches"],
                          "stages": mplan.exec_info()["stages"]}
         del msess, mplan
+        splan, ssess, scfg = build_swin(local)
+        ts = time_steps(ssess, 10, 3, flush, stream)
+        _, tf, _ = peaks()
+        slat = statistics.median(ts) * 1e3
+        si = splan.exec_info()
+        extra["swin"] = {"workload": "Swin-B 224x224 (torchvision swin_b), batch 1 per GPU (bf16 GEMM operands)",
+                         "latency_us": slat, "images_per_s": 1e6 / slat, "launches": si["launches"],
+                         "stages": si["stages"], "grid_barriers": si["barriers"],
+                         "tensor_frac": SWIN_FLOPS / (slat * 1e-6) / 1e12 / tf,
+                         "lowering": "generic fused-subprogram executor (exec.cu)"}
+        del ssess, splan
 
     if rank == 0:
         hbm, tf, src = peaks()

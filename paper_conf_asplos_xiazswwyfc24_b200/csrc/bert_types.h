@@ -34,7 +34,7 @@ enum {
   B_SMEM = B_CTRL_BYTES + BW_SLOTS * BW_SLOT_BYTES + B_AREGION + 1024   // + alignment slack
 };
 
-struct BStage {
+struct alignas(16) BStage {
   int32_t kind, ntasks, layer, idx;   // idx: position in the stage list
   // ---- GEMM: task = tile * nsplit + split; each split covers kchunks chunks of 64 along K
   int32_t nt, tiles_n, nsplit, kchunks;
@@ -48,8 +48,16 @@ struct BStage {
   int32_t qkmap, vtmap, d, H;
   uint16_t* ctx;                // bf16 [S][H], head h at columns h*64 ..
   float scale, eps;
+  // ---- point-to-point dependencies (instead of a grid barrier; §6.4 only needs a global sync for
+  // one-relies-on-many edges).  A consumer stage with fwait waits until flag fin[idx] reaches fneed
+  // (idx = head for ATTN, K split for a GEMM); a producer stage with fout adds 1 to
+  // fout[(n0 % fmod) / fdiv] after its epilogue.  Flags are 128 B apart.  arrive: the next stage
+  // waits on this stage's grid barrier.
+  int32_t fwait, fneed, fdiv, fmod;
+  unsigned int* fin;
+  unsigned int* fout;
   // ---- ROW: mode 0 convert (out_b = bf16(in)); mode 1 LayerNorm(sum_s part[s] + bias + res)
-  int32_t row_mode, cols, r_nsplit, pad1;
+  int32_t row_mode, cols, r_nsplit, arrive;
   const float* r_in;            // mode 0: fp32 [S][cols]; mode 1: partials [r_nsplit][S][cols]
   const float* r_bias;
   const float* r_res;
@@ -57,17 +65,17 @@ struct BStage {
   const float* r_beta;
   float* r_out_f;
   uint16_t* r_out_b;
-  int64_t pad2;
 };
 
 struct BertParams {
   const BStage* stages;
   const void* tmaps;            // CUtensorMap[] (128 B each)
-  unsigned int* ctrl;           // [0, nstages): per-barrier arrival counters; [nstages]: exit counter
+  unsigned int* ctrl;           // [0, nstages): per-barrier arrival counters; [nstages]: exit counter;
+                                // [nstages + 1 + 32 k]: point-to-point flag k (nflags of them)
   unsigned long long* prof;     // optional per-stage %globaltimer marks, null if off
   int32_t nstages, S;
   int32_t dbg_skip;             // debug: bit k set -> stages of kind k do no work (barriers only)
-  int32_t pad;
+  int32_t nflags;
 };
 
 }  // namespace souffle

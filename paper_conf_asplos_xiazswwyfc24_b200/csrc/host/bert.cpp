@@ -236,6 +236,7 @@ void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   bp.num_sms = dev.num_sms > 0 ? dev.num_sms : 148;
   const int sms = bp.num_sms;
   if (bp.S % 8) return no("S must be a multiple of 8 (V^T rows are TMA-loaded)");
+  if (bp.H > 768) return no("hidden size must be <= 768 (LayerNorm row stage: 3 columns per thread)");
   bp.qkv = full_cfg(3LL * bp.H, bp.H, sms, 64, "SOUFFLE_BERT_QKV");     // tiles never straddle a head
   // out-projection fused into attention: split-K over heads (K = 64 per head), N tiles of nt rows
   bp.out = BertGemmCfg{};
@@ -249,7 +250,8 @@ void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   bp.nstages = 1 + 6 * (int)bp.layers.size();
   // ---- workspace layout
   int64_t o = 0;
-  bp.o_ctrl = o; o = al(o + 4 * (bp.nstages + 2), 256);
+  bp.nflags = (int)bp.layers.size() * (bp.heads + bp.ffn2.nsplit);
+  bp.o_ctrl = o; o = al(o + 4 * (bp.nstages + 2 + 32 * (int64_t)bp.nflags), 256);
   bp.o_prof = o; o = al(o + 8 * (17 * bp.nstages + 2), 256);
   bp.o_stages = o; o = al(o + (int64_t)sizeof(BStage) * bp.nstages, 256);
   bp.o_tmaps = o; o = al(o + 128 * (kActMaps + 6 * (int64_t)bp.layers.size()), 256);
@@ -381,6 +383,15 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
   uint16_t* vt = (uint16_t*)(base + bp.o_vt);
   const float* X = (const float*)ptr(bp.X);
   float* Y = (float*)ptr(bp.Y);
+  unsigned* ctrl = (unsigned*)(base + bp.o_ctrl);
+  // point-to-point flags instead of the grid barriers QKV -> attention (head h reads only the Q/K/V tiles
+  // of head h) and FFN1 -> FFN2 (K split s reads only the FFN1 tiles of its K range).  Opt-in
+  // (SOUFFLE_BERT_P2P=1): measured on B200 the producer's release (fence + red, ~1 us after its
+  // stores) plus the consumer's acquire poll costs as much as the 148-CTA barrier, because all
+  // producers of a stage finish within ~0.2 us of each other.
+  const bool nop2p = std::getenv("SOUFFLE_BERT_P2P") == nullptr;
+  const bool p2p_qkv = !nop2p && bp.d % bp.qkv.nt == 0;
+  const bool p2p_ffn = !nop2p && (bp.ffn2.kchunks * 64) % bp.ffn1.nt == 0 && F % (bp.ffn2.kchunks * 64) == 0;
   std::vector<BStage> st;
   auto stage = [&](int kind, int layer) {
     BStage s;
@@ -419,7 +430,11 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
     a.bias = cptr(L.bq);   // bq, bk, bv are packed contiguously: the [Q | K | V] bias
     a.out_b = qk; a.out_vt = vt;
     st.push_back(a);
+    unsigned* fl_qkv = ctrl + bp.nstages + 1 + 32 * (l * (bp.heads + bp.ffn2.nsplit));
+    unsigned* fl_ffn = fl_qkv + 32 * bp.heads;
+    if (p2p_qkv) { st.back().fout = fl_qkv; st.back().fdiv = bp.d; st.back().fmod = (int)H; }   // the QKV stage
     BStage at = stage(BS_ATTN, l);
+    if (p2p_qkv) { at.fwait = 1; at.fin = fl_qkv; at.fneed = 3 * (bp.d / bp.qkv.nt); }
     at.heads = bp.heads; at.d = bp.d; at.H = (int)H;
     at.qkmap = MAP_QK; at.vtmap = MAP_VT;
     at.scale = (float)(1.0 / std::sqrt((double)bp.d));
@@ -431,9 +446,11 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
     st.push_back(ln(l, part_o, bp.out.nsplit, cptr(L.bo), xin, cptr(L.g1), cptr(L.be1), l1f, l1b));
     BStage f1 = gemm(l, bp.ffn1, F, H, t + 4, F, MAP_L1B, EP_GELU);
     f1.bias = cptr(L.c1); f1.out_b = hb;
+    if (p2p_ffn) { f1.fout = fl_ffn; f1.fdiv = bp.ffn2.kchunks * 64; f1.fmod = (int)F; }
     st.push_back(f1);
     BStage f2 = gemm(l, bp.ffn2, H, F, t + 5, H, MAP_H, EP_PARTIAL);
     f2.part = part_2;
+    if (p2p_ffn) { f2.fwait = 1; f2.fin = fl_ffn; f2.fneed = bp.ffn2.kchunks * 64 / bp.ffn1.nt; }
     st.push_back(f2);
     const bool last = l == nl - 1;
     st.push_back(ln(l, part_2, bp.ffn2.nsplit, cptr(L.c2), l1f, cptr(L.g2), cptr(L.be2), last ? Y : xf,
@@ -445,6 +462,7 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
     // barrier arrivals = CTAs with work (must match has_work() in kernels/bert.cu)
     st[i].workers = st[i].kind == BS_ROW ? std::min(bp.S, bp.num_sms) : st[i].ntasks;
   }
+  for (int i = 0; i + 1 < (int)st.size(); ++i) st[i].arrive = st[i + 1].fwait ? 0 : 1;
   cudaStream_t s = (cudaStream_t)stream;
   cudaError_t e = cudaMemsetAsync(base, 0, (size_t)bp.total, s);
   if (e == cudaSuccess)
@@ -487,6 +505,7 @@ souffle_status bert_run(Plan& p, void* ws, void* stream) {
   prm.ctrl = (unsigned*)(base + bp.o_ctrl);
   prm.prof = p.profiling ? (unsigned long long*)(base + bp.o_prof) : nullptr;
   prm.nstages = bp.nstages;
+  prm.nflags = bp.nflags;
   prm.S = bp.S;
   if (const char* dbg = std::getenv("SOUFFLE_BERT_DBG_SKIP")) prm.dbg_skip = std::atoi(dbg);   // timing studies
   cudaError_t e = bert_launch(prm, grid, (cudaStream_t)stream);

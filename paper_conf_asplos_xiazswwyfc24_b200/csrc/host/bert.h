@@ -34,6 +34,7 @@ struct BertPlan {
   BertGemmCfg qkv, out, ffn1, ffn2;
   int num_sms = 0;
   int nstages = 0;
+  int nflags = 0;                 // point-to-point flags in the control block (kernels/bert.cu)
   // workspace layout (byte offsets from the workspace base)
   int64_t o_ctrl = 0, o_stages = 0, o_tmaps = 0, o_prof = 0;
   int64_t o_xb = 0, o_ctx = 0, o_l1b = 0, o_l1f = 0, o_xf = 0;

@@ -82,6 +82,17 @@ __device__ __forceinline__ void submark(const BertParams& P, const BStage& st, i
   }
 }
 
+// watchdog for the spin waits: a dependency that never resolves (a planner bug) aborts the launch with
+// an error after ~2 s instead of hanging the GPU
+__device__ __forceinline__ void spin_guard(uint32_t& n, unsigned long long& t0) {
+  if ((++n & 1023u) == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t0 == 0) t0 = t;
+    else if (t - t0 > 2000000000ull) __trap();
+  }
+}
+
 // ------------------------------------------------------------------ grid barrier (split phase)
 __device__ __forceinline__ void grid_arrive(const BertParams& P, int k) {
   ptx::fence_proxy_async();   // generic-proxy writes of this stage -> TMA reads of later stages
@@ -94,8 +105,31 @@ __device__ __forceinline__ void grid_arrive(const BertParams& P, int k) {
 __device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target_arrivals) {
   if (threadIdx.x == 0) {
     const unsigned target = (unsigned)target_arrivals;
-    while (ptx::ld_acquire(&P.ctrl[k]) < target) {
-    }
+    uint32_t n = 0;
+    unsigned long long t0 = 0;
+    while (ptx::ld_acquire(&P.ctrl[k]) < target) spin_guard(n, t0);
+    ptx::fence_proxy_async();
+  }
+  csync();
+}
+
+// point-to-point dependency: the producer CTA publishes its epilogue stores (generic proxy -> the
+// consumer's TMA reads) and bumps one flag; the consumer polls only the flag of the data it reads
+__device__ __forceinline__ void flag_signal(const BStage& st, int n0) {
+  ptx::fence_proxy_async();
+  csync();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    unsigned* f = st.fout + 32 * ((n0 % st.fmod) / st.fdiv);
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(f), "r"(1u) : "memory");
+  }
+}
+__device__ __forceinline__ void flag_wait(const BStage& st, int idx) {
+  if (threadIdx.x == 0) {
+    const unsigned* f = st.fin + 32 * idx;
+    uint32_t n = 0;
+    unsigned long long t0 = 0;
+    while (ptx::ld_acquire(f) < (unsigned)st.fneed) spin_guard(n, t0);
     ptx::fence_proxy_async();
   }
   csync();
@@ -307,6 +341,7 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
     default: gemm_epilogue<64>(P, st, C, areg, n0, split); break;
   }
   if (tid == 0) submark(P, st, 4);
+  if (st.fout) flag_signal(st, n0);
 }
 
 // ------------------------------------------------------------------ attention stage
@@ -454,14 +489,24 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
 }
 
 // ------------------------------------------------------------------ row stage (one CTA per row)
-__device__ __forceinline__ float block_sum(Ctrl* C, int k, float x) {
+// one fused block reduction of (sum v, sum v^2)
+__device__ __forceinline__ float2 block_sum2(Ctrl* C, float2 x) {
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-  if ((threadIdx.x & 31) == 0) C->red[k][threadIdx.x >> 5] = x;
+  for (int o = 16; o > 0; o >>= 1) {
+    x.x += __shfl_xor_sync(0xffffffffu, x.x, o);
+    x.y += __shfl_xor_sync(0xffffffffu, x.y, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    C->red[0][threadIdx.x >> 5] = x.x;
+    C->red[1][threadIdx.x >> 5] = x.y;
+  }
   csync();
-  float s = 0.f;
+  float2 s = make_float2(0.f, 0.f);
 #pragma unroll
-  for (int w = 0; w < 8; ++w) s += C->red[k][w];
+  for (int w = 0; w < 8; ++w) {
+    s.x += C->red[0][w];
+    s.y += C->red[1][w];
+  }
   return s;
 }
 
@@ -504,15 +549,15 @@ __device__ void run_row(const BertParams& P, const BStage& st, Ctrl* C) {
       v[i] += a;
     }
     if (tid == 0) submark(P, st, 0);
-    float s = 0.f;
+    float2 sq = make_float2(0.f, 0.f);
 #pragma unroll
-    for (int i = 0; i < kRowPer; ++i) s += v[i];   // out-of-range columns hold 0
-    const float mu = block_sum(C, 0, s) / (float)cols;
-    float q = 0.f;
-#pragma unroll
-    for (int i = 0; i < kRowPer; ++i)
-      if (tid + 256 * i < cols) q += (v[i] - mu) * (v[i] - mu);
-    const float var = block_sum(C, 1, q) / (float)cols;
+    for (int i = 0; i < kRowPer; ++i) {   // out-of-range columns hold 0
+      sq.x += v[i];
+      sq.y += v[i] * v[i];
+    }
+    sq = block_sum2(C, sq);   // one-pass statistics (R10): one barrier instead of two
+    const float mu = sq.x / (float)cols;
+    const float var = fmaxf(sq.y / (float)cols - mu * mu, 0.f);
     const float rs = rsqrtf(var + st.eps);
     if (tid == 0) submark(P, st, 1);
 #pragma unroll
@@ -592,7 +637,10 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
   for (int s = 0; s < P.nstages; ++s) {
     const BStage& st = sbuf[s & 1];
     const bool work = has_work(P, st);
-    if (work && s > 0) grid_wait(P, s - 1, prev_workers);
+    if (work && s > 0) {
+      if (st.fwait) flag_wait(st, st.kind == BS_ATTN ? (int)blockIdx.x % st.heads : (int)blockIdx.x % st.nsplit);
+      else grid_wait(P, s - 1, prev_workers);
+    }
     prev_workers = st.workers;
     if (s + 1 < P.nstages && tid < (int)(sizeof(BStage) / 16))
       reinterpret_cast<int4*>(sbuf + ((s + 1) & 1))[tid] = __ldg(reinterpret_cast<const int4*>(P.stages + s + 1) + tid);
@@ -618,7 +666,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
         }
       }
       if (tid == 0) submark(P, st, 6);
-      if (s + 1 < P.nstages) grid_arrive(P, s);
+      if (st.arrive) grid_arrive(P, s);
       if (tid == 0) submark(P, st, 7);
     }
     csync();   // descriptor s+1 visible; everyone is done with descriptor s
@@ -631,6 +679,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
     if (old == gridDim.x - 1) {
       __threadfence();
       for (int k = 0; k <= P.nstages; ++k) P.ctrl[k] = 0u;
+      for (int k = 0; k < P.nflags; ++k) P.ctrl[P.nstages + 1 + 32 * k] = 0u;
     }
   }
   if (P.prof && blockIdx.x == 0 && tid == 0) {
