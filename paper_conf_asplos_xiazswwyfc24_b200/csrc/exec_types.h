@@ -94,7 +94,8 @@ struct GemmMember {
   int32_t a_f32;            // TC manual path: Addr of fp32 A, rows contiguous with stride K
   int32_t acc_off;          // TC split-K: workspace float offset of the fp32 accumulator
   int32_t cnt_off;          // TC split-K: workspace u32 offset of per-tile arrival counters
-  int32_t pad;
+  int32_t gemv;             // SIMT: 1 -> skinny GEMM (few rows): a warp per output element,
+                            // lanes split K; task = 8 consecutive (row, col) outputs
 };
 
 struct Stage {

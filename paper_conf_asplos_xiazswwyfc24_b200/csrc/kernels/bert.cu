@@ -146,7 +146,11 @@ __device__ __forceinline__ bool has_work(const BertParams& P, const BStage& st) 
 // K-chunk order of a task: rotated by the CTA index so that the CTAs of a stage, which all read
 // the same activation tile, spread their concurrent A requests over all L2 slices instead of
 // hammering the lines of one chunk together (the accumulation order changes; the sum does not)
-__device__ __forceinline__ int rot_chunk(int i, int nk) { return (i + (int)blockIdx.x) % nk; }
+__device__ __forceinline__ int rot_chunk(const BertParams& P, int i, int nk) {
+  if (P.dbg_skip & 8192) return i;                                    // timing study: no rotation
+  if (P.dbg_skip & 16384) return (i + (int)blockIdx.x / 16) % nk;     // timing study: groups of 16 CTAs
+  return (i + (int)blockIdx.x) % nk;
+}
 
 // weight K-chunks per ring slot for an N tile of nt rows (16 KB / (nt * 128 B))
 __device__ __forceinline__ int wgroup(int nt) { return max(1, BW_SLOT_BYTES / (nt * 128)); }
@@ -179,7 +183,7 @@ __device__ void weight_producer(const BertParams& P, Ctrl* C, char* wring) {
       ptx::mbar_arrive_expect_tx(&C->wfull[slot], (uint32_t)(cnt * nt * 128));
       for (int j = 0; j < cnt; ++j)
         ptx::tma_load_2d(wring + slot * BW_SLOT_BYTES + j * nt * 128, tmaps + 128 * map, &C->wfull[slot],
-                         (kc0 + rot_chunk(c0 + j, nk)) * 64, row);
+                         (kc0 + rot_chunk(P, c0 + j, nk)) * 64, row);
     }
   }
 }
@@ -288,7 +292,7 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
       if (ms.aload >= BA_SLOTS) ptx::mbar_wait(&C->aempty[slot], ((ms.aload / BA_SLOTS) - 1) & 1);
       if (ptx::elect_one()) {
         ptx::mbar_arrive_expect_tx(&C->afull[slot], BA_SLOT_BYTES);
-        ptx::tma_load_2d(areg + slot * BA_SLOT_BYTES, amap, &C->afull[slot], (kc0 + rot_chunk(c, nk)) * 64, 0);
+        ptx::tma_load_2d(areg + slot * BA_SLOT_BYTES, amap, &C->afull[slot], (kc0 + rot_chunk(P, c, nk)) * 64, 0);
       }
       __syncwarp();
       ++ms.aload;

@@ -730,30 +730,45 @@ __device__ __noinline__ void run_ew(const Params& P, const Stage& st, char* smem
 }
 
 // ================================================================== REDUCE stage (warp per row)
+// Rows of at most 16 chunks (<= 128 columns, e.g. the 49-wide window-attention softmax rows of Swin)
+// are packed several per warp: a group of G lanes (a power of two >= the row's chunk count) owns one
+// row, so short rows do not leave most of the warp idle.
 __device__ __noinline__ void run_reduce(const Params& P, const Stage& st, char* smem) {
   const Prog pre = cached_prog(smem, 0);
   const Prog post = cached_prog(smem, 1);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float red[MAX_RED] = {0.f, 0.f, 0.f, 0.f};
-  for (int64_t o = (int64_t)blockIdx.x * 8 + warp; o < st.rows; o += (int64_t)gridDim.x * 8) {
+  const int chunks = (st.cols + CHUNK - 1) / CHUNK;
+  int G = 32;
+  if (chunks <= 16) {
+    G = 1;
+    while (G < chunks) G <<= 1;
+  }
+  const int rpw = 32 / G;                      // rows per warp
+  const int sub = lane / G, gl = lane % G;     // row slot within the warp, lane within the group
+  const int64_t rows_per_cta = 8 * rpw;
+  for (int64_t ob = (int64_t)blockIdx.x * rows_per_cta + warp * rpw; ob < st.rows; ob += (int64_t)gridDim.x * rows_per_cta) {
+    const int64_t o = ob + sub;
+    const bool live = o < st.rows;
     float acc = st.red_fn ? -INFINITY : 0.f;
-    for (int64_t c0 = (int64_t)lane * CHUNK; c0 < st.cols; c0 += 32 * CHUNK) {
-      int nv = (int)((st.cols - c0) < CHUNK ? (st.cols - c0) : CHUNK);
-      float vals[CHUNK];
-      float zero[CHUNK] = {0, 0, 0, 0, 0, 0, 0, 0};
-      float dummy[MAX_RED] = {0.f, 0.f, 0.f, 0.f};
-      run_prog<CHUNK>(P, pre, o, c0, nv, zero, dummy, vals);
+    if (live) {
+      for (int64_t c0 = (int64_t)gl * CHUNK; c0 < st.cols; c0 += (int64_t)G * CHUNK) {
+        int nv = (int)((st.cols - c0) < CHUNK ? (st.cols - c0) : CHUNK);
+        float vals[CHUNK];
+        float zero[CHUNK] = {0, 0, 0, 0, 0, 0, 0, 0};
+        float dummy[MAX_RED] = {0.f, 0.f, 0.f, 0.f};
+        run_prog<CHUNK>(P, pre, o, c0, nv, zero, dummy, vals);
 #pragma unroll
-      for (int j = 0; j < CHUNK; ++j)
-        if (j < nv) acc = st.red_fn ? fmaxf(acc, vals[j]) : acc + vals[j];
+        for (int j = 0; j < CHUNK; ++j)
+          if (j < nv) acc = st.red_fn ? fmaxf(acc, vals[j]) : acc + vals[j];
+      }
     }
-#pragma unroll
-    for (int s = 16; s > 0; s >>= 1) {
-      float y = __shfl_xor_sync(0xffffffffu, acc, s);
+    for (int s2 = G >> 1; s2 > 0; s2 >>= 1) {
+      float y = __shfl_xor_sync(0xffffffffu, acc, s2);
       acc = st.red_fn ? fmaxf(acc, y) : acc + y;
     }
     acc *= st.red_scale;
-    if (lane == 0) {
+    if (live && gl == 0) {
       float a1[1] = {acc};
       run_prog<1>(P, post, o, 0, 1, a1, red);
       flush_reds(P, post, o, red);
@@ -783,6 +798,39 @@ __device__ __noinline__ void run_gemm_simt(const Params& P, const Stage& st, cha
       cur = mi;
     }
     const int local = task - M.task0;
+    if (M.gemv) {
+      // skinny GEMM (e.g. a classifier head on one pooled row): warp w computes output 8 * task + w,
+      // lanes stride over K (coalesced rows of B), shuffle reduction, lane 0 runs the chain
+      const Addr A = P.addrs[M.a_addr];
+      const Addr B = P.addrs[M.b_addr];
+      const int warp = tid >> 5, lane = tid & 31;
+      const int64_t rows = (int64_t)M.batch * M.M;
+      for (int i = 0; i < 1; ++i) {
+        const int64_t idx = (int64_t)local * 8 + warp;
+        const int64_t r = idx / M.N;
+        const int n = (int)(idx % M.N);
+        if (r >= rows) break;
+        const int64_t b = r / M.M;
+        float acc = 0.f;
+        for (int k = lane; k < M.K; k += 32) {
+          float a = ld1(P, A, addr_off(P, A, r, k));
+          float bb = ld1(P, B, addr_off(P, B, b * M.N + n, k));
+          if (M.prec) {
+            a = __bfloat162float(__float2bfloat16_rn(a));
+            bb = __bfloat162float(__float2bfloat16_rn(bb));
+          }
+          acc = fmaf(a, bb, acc);
+        }
+#pragma unroll
+        for (int s2 = 16; s2 > 0; s2 >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, s2);
+        if (lane == 0) {
+          float a1[1] = {acc};
+          run_prog<1>(P, G, r, n, 1, a1, red);
+          flush_reds(P, G, r, red);
+        }
+      }
+      continue;
+    }
     const int tmi = local / M.tiles_n, tn = local % M.tiles_n;
     const int mt = (M.M + 63) / 64;
     const int b = tmi / mt, tm = tmi % mt;
