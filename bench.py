@@ -293,14 +293,19 @@ def main():
     clk = Clocks(local) if rank == 0 else None
     times = time_steps(sess, args.steps, args.warmup, flush, stream, clk)
     clocks = clk.stop() if clk else None
-    total_ms = sum(times)
+    from paper_conf_asplos_xiazswwyfc24_b200 import replicas as R
+    total_ms = R.max_over_ranks(sum(times), dev)          # the job's time is the slowest replica's
     if ws > 1:
-        t = torch.tensor([total_ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
         dist.barrier()
     ms_per_step = total_ms / args.steps
-    value = ws * args.steps / (total_ms / 1e3)
+    value = R.aggregate_rate(args.steps, total_ms / 1e3)  # inferences of all ranks / max time
+    # after timing: gather every replica's output to rank 0 over NCCL (the only collective) and check
+    # the replicas agree (same request -> same result; the oracle check itself is in tests/)
+    gathered = R.gather_to_rank0(sess.outputs[y])
+    replica_check = None
+    if gathered is not None:
+        replica_check = {"replicas": int(gathered.shape[0]),
+                         "max_abs_diff_vs_rank0": float((gathered - gathered[0:1]).abs().max().item())}
 
     # ---- e2e through the public API with host buffers (H2D input, D2H output inside the timed region)
     xin = torch.from_numpy(np.ascontiguousarray(x_host, dtype=np.float32)).pin_memory()
@@ -322,11 +327,7 @@ def main():
         b.record(stream)
         b.synchronize()
         e_ms.append(a.elapsed_time(b))
-    e_total = sum(e_ms)
-    if ws > 1:
-        t = torch.tensor([e_total], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e_total = float(t.item())
+    e_total = R.max_over_ranks(sum(e_ms), dev)
 
     extra = {}
     if rank == 0 and not args.no_v0:
@@ -392,7 +393,8 @@ def main():
                          "traffic": traffic, "peak_source": src,
                          "algorithmic_bytes_per_launch": ALGO_BYTES,
                          "tensor_frac": ALGO_FLOPS / (med * 1e-3) / 1e12 / tf},
-            "e2e": {"value": ws * args.steps / (e_total / 1e3), "unit": "inferences/s",
+            "replica_check": replica_check,
+            "e2e": {"value": R.aggregate_rate(args.steps, e_total / 1e3), "unit": "inferences/s",
                     "h2d_bytes_per_step": int(xin.numel() * 4), "d2h_bytes_per_step": int(yout.numel() * 4)},
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks,
