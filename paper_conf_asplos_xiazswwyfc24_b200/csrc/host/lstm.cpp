@@ -126,13 +126,19 @@ void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   if (g.outputs != expect) return no("outputs are not [top_t..., (h_n, c_n) per layer]");
   lp.hn = h;
   lp.cn = cc;
-  // ---- resources: 32 hidden units (128 gate rows) per CTA, weights resident in shared memory
-  if (lp.H % 32 || lp.I % 8) return no("needs H % 32 == 0 and I % 8 == 0");
-  lp.NP = lp.H / 32;
-  if (2 * lp.NP > 32) return no("more than 16 CTAs per layer");
+  // ---- resources: NP CTAs per layer, each owning <= 32 hidden units (<= 128 gate rows) whose
+  // weights stay resident in shared memory.  The per-step GEMV is bound by reading those weights
+  // from shared memory, so NP is as large as the SMs allow (all layers' CTAs co-resident).
+  if (lp.H % 8 || lp.I % 8) return no("needs H % 8 == 0 and I % 8 == 0");
+  const int sms = dev.num_sms > 0 ? dev.num_sms : 148;
+  const int np_min = (lp.H + LSTM_UNITS - 1) / LSTM_UNITS;
+  lp.NP = std::max(np_min, std::min(sms / lp.L, lp.H / 8));
+  if (const char* e = std::getenv("SOUFFLE_LSTM_NP")) {   // timing studies
+    const int v = std::atoi(e);
+    if (v >= np_min && v * lp.L <= sms && v <= lp.H) lp.NP = v;
+  }
   lp.K_max = std::max(lp.I, lp.H) + lp.H;
   if (lp.K_max > 2 * LSTM_THREADS) return no("input + hidden width above 1024");
-  const int sms = dev.num_sms > 0 ? dev.num_sms : 148;
   if (lp.L * lp.NP > sms) return no("more CTAs than SMs");
   if (lstm_smem_bytes(lp.K_max, lp.w_f32) > (size_t)LSTM_MAX_SMEM) return no("weights of 32 units do not fit shared memory");
   int64_t o = 0;
@@ -153,7 +159,7 @@ std::string lstm_describe(const LstmPlan& lp) {
   }
   os << "pattern lstm: " << lp.L << " layers x " << lp.T << " steps, H=" << lp.H << " I=" << lp.I << " ("
      << (lp.w_f32 ? "fp32" : "bf16") << " weights) -> 1 persistent launch (kernels/lstm.cu), " << lp.L * lp.NP
-     << " CTAs = " << lp.NP << " per layer x 32 units, weights resident in shared memory, wavefront of "
+     << " CTAs = " << lp.NP << " per layer x <= 32 units, weights resident in shared memory, wavefront of "
      << lp.L + lp.T - 1 << " dependent steps synchronised through tagged (value, step) words\n";
   return os.str();
 }

@@ -1,7 +1,9 @@
 // Persistent wavefront LSTM kernel for sm_100a (§8.4; Fig. 7).
 //
-// One cooperative launch runs the whole stacked LSTM (L layers x T steps).  CTA (l, p) owns hidden
-// units [32p, 32p+32) of layer l: the 128 gate rows (i, f, g, o of those units) of [W_ih | W_hh] are
+// One cooperative launch runs the whole stacked LSTM (L layers x T steps).  CTA (l, p) owns nu <= 32
+// hidden units [u0, u0 + nu) of layer l (u0 = p H / NP; NP CTAs per layer, as many as the SMs allow,
+// so that the per-step GEMV -- bound by reading the CTA's weights from shared memory -- is spread
+// over all SMs): the 4 nu gate rows (i, f, g, o of those units) of [W_ih | W_hh] are
 // loaded into shared memory ONCE and reused for all T steps (the paper's "weights stay on chip";
 // HBM reads the 10.5 MB of bf16 weights once instead of once per step).  Per step:
 //   wait   h(l, t-1) and h(l-1, t) are read as (value, tag) words straight from L2, spinning until
@@ -47,6 +49,8 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int l = blockIdx.x / P.NP, p = blockIdx.x % P.NP;
   const int H = P.H, T = P.T, NP = P.NP, Kst = P.K_max;
+  const int u0 = (p * H) / NP, nu = ((p + 1) * H) / NP - u0;   // this CTA's hidden units (nu <= 32)
+  const int R = 4 * nu;                                         // gate rows r = gate * nu + j
   const LstmLayer& Ly = P.layers[l];
   const int I = Ly.in_dim, K = I + H;
   constexpr int ES = F32 ? 4 : 2;
@@ -60,19 +64,21 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
     const int vpr = K * ES / 16;   // 16-byte vectors per row
     for (int e = tid; e < LSTM_ROWS * vpr; e += LSTM_THREADS) {
       const int r = e / vpr, v = e % vpr;
-      const int grow = (r >> 5) * H + p * LSTM_UNITS + (r & 31);
+      if (r >= R) break;
+      const int grow = (r / nu) * H + u0 + (r % nu);
       const int col = v * 16 / ES;   // first element of this vector
       const char* src = col < I ? (const char*)Ly.W + ((int64_t)grow * I + col) * ES
                                 : (const char*)Ly.U + ((int64_t)grow * H + (col - I)) * ES;
       *reinterpret_cast<uint4*>(w + ((int64_t)r * Kst + col) * ES) = __ldg(reinterpret_cast<const uint4*>(src));
     }
-    for (int r = tid; r < LSTM_ROWS; r += LSTM_THREADS) {
-      const int grow = (r >> 5) * H + p * LSTM_UNITS + (r & 31);
+    for (int r = tid; r < R; r += LSTM_THREADS) {
+      const int grow = (r / nu) * H + u0 + (r % nu);
       bias[r] = __ldg(Ly.b_ih + grow) + __ldg(Ly.b_hh + grow);
     }
   }
-  const int unit = p * LSTM_UNITS + lane;
-  float c = (warp == 0) ? __ldg(Ly.c0 + unit) : 0.f;
+  const int unit = u0 + lane;
+  const bool own = lane < nu;
+  float c = (warp == 0 && own) ? __ldg(Ly.c0 + unit) : 0.f;
   float h = 0.f;
   __syncthreads();
 
@@ -120,8 +126,9 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
     }
     __syncthreads();
     stamp(t, 1);
-    // ---- gates: warp w computes rows RPW*w ..; lanes split the K columns in groups of 8
-    {
+    // ---- gates: warp w computes rows RPW*w ..; lanes split the K columns in groups of 8 (warps
+    // beyond the CTA's 4 nu rows skip: the smem weight reads are the step's bound)
+    if (warp * 8 < R) {
       constexpr int RPW = LSTM_ROWS / (LSTM_THREADS / 32);   // rows per warp (8 with 16 warps)
       static_assert(RPW == 8, "reduction below assumes 8 rows per warp");
       float acc[RPW];
@@ -167,11 +174,11 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
     __syncthreads();
     stamp(t, 2);
     // ---- cell update (warp 0, one unit per lane) and publication of h(l, t)
-    if (warp == 0) {
+    if (warp == 0 && own) {
       const float gi = gates[lane] + bias[lane];
-      const float gf = gates[32 + lane] + bias[32 + lane];
-      const float gg = gates[64 + lane] + bias[64 + lane];
-      const float go = gates[96 + lane] + bias[96 + lane];
+      const float gf = gates[nu + lane] + bias[nu + lane];
+      const float gg = gates[2 * nu + lane] + bias[2 * nu + lane];
+      const float go = gates[3 * nu + lane] + bias[3 * nu + lane];
       c = sigm(gf) * c + sigm(gi) * tanhf(gg);
       h = sigm(go) * tanhf(c);
       if (l == P.L - 1) P.top[t][unit] = h;
@@ -180,7 +187,7 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
       asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(dst), "l"(w64) : "memory");
     }
   }
-  if (warp == 0) {
+  if (warp == 0 && own) {
     Ly.h_n[unit] = h;
     Ly.c_n[unit] = c;
   }
