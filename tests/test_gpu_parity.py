@@ -184,3 +184,36 @@ def test_lstm_full_config_bf16_weights():
     assert "pattern lstm: 10 layers x 100 steps" in plan.describe()
     assert rel_err(gt, wt) <= 1e-4, rel_err(gt, wt)
     assert rel_err(gs, ws) <= 1e-4
+
+
+@pytest.mark.parametrize("seq,hidden,heads,ffn,layers", [
+    (72, 768, 12, 3072, 2),     # ragged: 72 of the 128 rows of the M tile, masked softmax keys
+    (8, 256, 4, 1024, 3),       # minimum multiple of 8 tokens, 4 heads, smaller FFN
+    (128, 384, 6, 1536, 2),     # 6 heads: different tile counts in every stage
+])
+def test_bert_pattern_ragged_shapes(seq, hidden, heads, ffn, layers):
+    """The persistent BERT kernel on shapes other than BERT-base (edge cases of its tile policy)."""
+    cfg = dict(synth.BERT_BASE, seq=seq, hidden=hidden, heads=heads, ffn=ffn, layers=layers)
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    emu = te.evaluate(spec, og.bert_feed(X, plist, x, w), bf16_operands=True)[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    (out,), plan = run(g, og.bert_feed(gX, gpl, x, w), [gy])
+    assert "pattern bert:" in plan.describe() and "not used" not in plan.describe().splitlines()[0]
+    err = float(np.abs(out - emu).max())
+    assert err <= 2e-2, (err, plan.describe())
+
+
+def test_bert_seq_not_multiple_of_8_runs_generic():
+    """S = 20 is outside the pattern kernel (V^T rows are TMA-loaded in 8s): the generic fused
+    executor runs it, still matching the oracle."""
+    cfg = dict(synth.BERT_BASE, seq=20, hidden=128, heads=2, ffn=512, layers=1)
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    emu = te.evaluate(spec, og.bert_feed(X, plist, x, w), bf16_operands=True)[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    (out,), plan = run(g, og.bert_feed(gX, gpl, x, w), [gy])
+    assert "not used" in plan.describe().splitlines()[0]
+    assert float(np.abs(out - emu).max()) <= 2e-2
