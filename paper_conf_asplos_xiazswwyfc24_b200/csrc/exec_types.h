@@ -110,7 +110,7 @@ struct Stage {
   int32_t at_B, at_S, at_d, at_q, at_k, at_v;  // q/k/v: Addr index (base, buf used)
   float at_scale;
   int32_t barrier_after;            // the next stage of the same launch starts with a grid barrier
-  int32_t pad[2];
+  int32_t at_add[2];                // ATTN: Addr of additive score terms at (b*S + i, j), -1 if none
 };
 
 struct Launch {

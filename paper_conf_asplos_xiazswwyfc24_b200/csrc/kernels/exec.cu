@@ -1122,25 +1122,29 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
   for (int b = blockIdx.x; b < st.at_B; b += gridDim.x) {
     if (tid == 0) mark(P, ctl, 0);
     const int64_t hb = (int64_t)b * S * d;
-    // ---- stage Q, K (K-major, swizzled) and V^T
-    const int chunks = 128 * (d / 8);
+    // ---- stage Q, K (K-major, swizzled; head dim zero-padded to dk = 64 / 128 so every row is whole
+    // 128-byte swizzle atoms) and V^T
+    const int dk = (d + 63) & ~63;
+    const int chunks = 128 * (dk / 8);
     for (int e = tid; e < chunks; e += kThreads) {
-      int s = e / (d / 8), c8 = e % (d / 8);
+      int s = e / (dk / 8), c8 = e % (dk / 8);
       int atom = c8 / 8, cb = (c8 % 8) * 16;
       uint4 qv = make_uint4(0, 0, 0, 0), kv = make_uint4(0, 0, 0, 0), vv = make_uint4(0, 0, 0, 0);
-      if (s < S) {
+      if (s < S && c8 * 8 < d) {
         qv = __ldcg(reinterpret_cast<const uint4*>(gq + hb + (int64_t)s * d + c8 * 8));
         kv = __ldcg(reinterpret_cast<const uint4*>(gk + hb + (int64_t)s * d + c8 * 8));
         vv = __ldcg(reinterpret_cast<const uint4*>(gv + hb + (int64_t)s * d + c8 * 8));
       }
       *reinterpret_cast<uint4*>(Qs + atom * 16384 + sw128(s, cb)) = qv;
       *reinterpret_cast<uint4*>(Ks + atom * 16384 + sw128(s, cb)) = kv;
-      const uint16_t* vp = reinterpret_cast<const uint16_t*>(&vv);
-      int katom = s / 64, kb = (s % 64) * 2;
+      if (c8 * 8 < d) {
+        const uint16_t* vp = reinterpret_cast<const uint16_t*>(&vv);
+        int katom = s / 64, kb = (s % 64) * 2;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        int dd = c8 * 8 + j;
-        *reinterpret_cast<uint16_t*>(Vt + katom * (d * 128) + sw128(dd, kb)) = vp[j];
+        for (int j = 0; j < 8; ++j) {
+          int dd = c8 * 8 + j;
+          *reinterpret_cast<uint16_t*>(Vt + katom * (d * 128) + sw128(dd, kb)) = vp[j];
+        }
       }
     }
     ptx::fence_proxy_async();
@@ -1151,7 +1155,7 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
       ptx::tc_fence_after();
       const uint32_t idesc = ptx::idesc_bf16(128, 128);
       const uint32_t q0 = ptx::smem_u32(Qs), k0 = ptx::smem_u32(Ks);
-      for (int ks = 0; ks < d / 16; ++ks) {
+      for (int ks = 0; ks < dk / 16; ++ks) {
         uint32_t off = (ks / 4) * 16384 + (ks % 4) * 32;
         ptx::mma_bf16(ctl->tmem_base, ptx::sdesc_sw128(q0 + off), ptx::sdesc_sw128(k0 + off), idesc, ks > 0);
       }
@@ -1168,13 +1172,48 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
       // three cheap passes over TMEM (16 columns at a time) keep the register footprint small
       const uint32_t tb = ctl->tmem_base + ((uint32_t)(q * 32) << 16) + half * 64;
       float mx = -INFINITY;
+      // additive score terms (e.g. relative-position bias, shifted-window mask): applied once, the
+      // scaled + biased scores are written back to TMEM and the later passes use scale 1
+      const bool adds = st.at_add[0] >= 0;
+      const int nadd = adds ? (st.at_add[1] >= 0 ? 2 : 1) : 0;
+      Addr AD[2];
+      if (adds) AD[0] = P.addrs[st.at_add[0]];
+      if (nadd > 1) AD[1] = P.addrs[st.at_add[1]];
+      const float sc1 = adds ? 1.f : scale;
 #pragma unroll 1
       for (int c0 = 0; c0 < 64; c0 += 16) {
+        if (half * 64 + c0 >= S) break;
         float v[16];
         ptx::tmem_ld16(tb + c0, v);
+        if (adds) {
+          const int64_t r = (int64_t)b * S + row;
+          float t[2][16];
+#pragma unroll
+          for (int k = 0; k < 2; ++k) {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) t[k][j] = 0.f;
+            if (k < nadd && row < S) {
+              // every load of the 16 columns is issued before any is used
+              const Addr& A = AD[k];
+              const int64_t rb = A.mode == 0 ? A.base + r * A.rs : A.mode == 1 ? A.base + P.tabs[A.rtab + r] : 0;
+#pragma unroll
+              for (int j = 0; j < 16; ++j) {
+                const int col = half * 64 + c0 + j;
+                if (col < S) {
+                  const int64_t o = A.mode == 0 ? rb + col * A.cs
+                                  : A.mode == 1 ? rb + P.tabs[A.ctab + col] : addr_off(P, A, r, col);
+                  t[k][j] = ld1(P, A, o);
+                }
+              }
+            }
+          }
+#pragma unroll
+          for (int j = 0; j < 16; ++j) v[j] = v[j] * scale + t[0][j] + t[1][j];
+          ptx::tmem_st16(tb + c0, v);
+        }
 #pragma unroll
         for (int j = 0; j < 16; ++j)
-          if (half * 64 + c0 + j < S) mx = fmaxf(mx, v[j] * scale);
+          if (half * 64 + c0 + j < S) mx = fmaxf(mx, v[j] * sc1);
       }
       float* xch = reinterpret_cast<float*>(Qs);    // [2][128] exchange (Q is consumed by now)
       xch[half * 128 + row] = mx;
@@ -1187,7 +1226,7 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
         ptx::tmem_ld16(tb + c0, v);
 #pragma unroll
         for (int j = 0; j < 16; ++j)   // ex2.approx (rel. err ~2^-22): P is rounded to bf16 anyway
-          if (half * 64 + c0 + j < S) z += __expf(v[j] * scale - mx);
+          if (half * 64 + c0 + j < S) z += __expf(v[j] * sc1 - mx);
       }
       __syncthreads();
       xch[half * 128 + row] = z;
@@ -1199,7 +1238,7 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
         float v[16];
         ptx::tmem_ld16(tb + c0, v);
 #pragma unroll
-        for (int j = 0; j < 16; ++j) v[j] = (half * 64 + c0 + j < S) ? __expf(v[j] * scale - mx) * iz : 0.f;
+        for (int j = 0; j < 16; ++j) v[j] = (half * 64 + c0 + j < S) ? __expf(v[j] * sc1 - mx) * iz : 0.f;
 #pragma unroll
         for (int h8 = 0; h8 < 16; h8 += 8) {
           uint32_t pk[4];
