@@ -44,7 +44,6 @@ struct Ctrl {
   uint32_t tmem_base;
   volatile int cur_stage;       // debug (dbg_skip bit 12): the producer does not run ahead of the executor
   float red[2][8];
-  float bias_s[128];            // the GEMM task's bias columns, staged by the idle warps during the mainloop
 };
 static_assert(sizeof(Ctrl) <= 1024, "control block");
 
@@ -217,10 +216,10 @@ __device__ __forceinline__ void gemm_epilogue(const BertParams& P, const BStage&
   else ptx::tmem_ld64(taddr, v);
   ptx::tc_fence_before();
   if (st.epi != EP_PARTIAL) {
-    const float4* bp = reinterpret_cast<const float4*>(C->bias_s + half * COLS);   // staged in run_gemm
+    const float4* bp = reinterpret_cast<const float4*>(st.bias + n0 + half * COLS);
 #pragma unroll
     for (int c = 0; c < COLS; c += 4) {
-      const float4 b = bp[c / 4];
+      const float4 b = __ldg(bp + c / 4);
       v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
     }
     if (st.epi == EP_GELU) {
@@ -334,15 +333,10 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
     if (tid == 0) submark(P, st, 2);    // all MMAs issued
   }
 
-  // ---- bias columns -> shared memory by the warps idle during the mainloop (the epilogue then never
-  // waits on an L2 round trip)
-  if (warp >= 2 && st.epi != EP_PARTIAL)
-    for (int i = tid - 64; i < nt; i += BERT_COMPUTE - 64) C->bias_s[i] = __ldg(st.bias + n0 + i);
   // ---- epilogue (all 8 warps: warp w reads TMEM lanes 32*(w%4).., column half w/4)
   ptx::mbar_wait(&C->accb, ms.accph);
   ms.accph ^= 1;
   ptx::tc_fence_after();
-  if (st.epi != EP_PARTIAL) csync();   // bias_s visible to every warp
   if (tid == 0) submark(P, st, 3);
   switch (nt) {
     case 16: gemm_epilogue<8>(P, st, C, areg, n0, split); break;
