@@ -217,3 +217,24 @@ def test_bert_seq_not_multiple_of_8_runs_generic():
     (out,), plan = run(g, og.bert_feed(gX, gpl, x, w), [gy])
     assert "not used" in plan.describe().splitlines()[0]
     assert float(np.abs(out - emu).max()) <= 2e-2
+
+
+def test_bert_pattern_repeated_launches_reuse_workspace():
+    """Three back-to-back launches on one workspace: the barrier counters are reset by the last CTA
+    of each launch, so every launch must reproduce the oracle (and the same bits up to atomics-free
+    determinism: the BERT kernel has no atomics on the data path)."""
+    cfg = dict(synth.BERT_BASE, layers=2)
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    emu = te.evaluate(spec, og.bert_feed(X, plist, x, w), bf16_operands=True)[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    plan = g.partition(L.device_query(0))
+    s = session(g, plan, og.bert_feed(gX, gpl, x, w), [gy])
+    outs = []
+    for _ in range(3):
+        s.run()
+        outs.append(s.result(gy))
+    for o in outs:
+        assert float(np.abs(o - emu).max()) <= 2e-2
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[1], outs[2])
