@@ -141,7 +141,8 @@ enum {
   SOUFFLE_FLAG_NO_VERTICAL = 4u,    /* disable §6.2 vertical transformation (materialise OR TEs)   */
   SOUFFLE_FLAG_NO_GLOBAL_SYNC = 8u, /* one launch per stage instead of grid barriers (§6.4)        */
   SOUFFLE_FLAG_NO_PREFETCH = 16u,   /* disable cross-stage weight prefetch (§6.5)                  */
-  SOUFFLE_FLAG_NO_LN_REWRITE = 32u  /* keep LayerNorm as two dependent reductions                  */
+  SOUFFLE_FLAG_NO_LN_REWRITE = 32u, /* keep LayerNorm as two dependent reductions                  */
+  SOUFFLE_FLAG_NO_PATTERN = 64u     /* generic lowering even where a model pattern kernel matches  */
 };
 /* Analyses the graph, partitions it and lowers every subprogram to a stage list.  Pure host
  * code.  `dev` may come from souffle_device_query or souffle_device_b200. */

@@ -15,6 +15,7 @@ EW = dict(add=0, sub=1, mul=2, div=3, max=4, exp=5, tanh=6, sigmoid=7, relu=8, g
 RED = dict(sum=0, max=1, mean=2)
 FLAG_UNFUSED, FLAG_NO_HORIZONTAL, FLAG_NO_VERTICAL, FLAG_NO_GLOBAL_SYNC, FLAG_NO_PREFETCH, FLAG_NO_LN_REWRITE = (
     1, 2, 4, 8, 16, 32)
+FLAG_NO_PATTERN = 64
 
 ERRORS = {1: "INVALID_ARG", 2: "SHAPE", 3: "UNSUPPORTED", 4: "RESOURCE", 5: "CUDA", 6: "STATE", 7: "OOM"}
 

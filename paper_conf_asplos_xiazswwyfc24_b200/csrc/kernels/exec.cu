@@ -794,6 +794,7 @@ __device__ __noinline__ void run_gemm_simt(const Params& P, const Stage& st, cha
     }
     const GemmMember& M = (mi == pf) ? ctrl_of(smem)->mem : P.members[st.mem0 + mi];
     if (mi != cur) {
+      __syncthreads();   // every warp is done with the previous member's program before it is replaced
       G = stage_prog(P, M.prog, cache_of(smem, 0));
       cur = mi;
     }
@@ -987,6 +988,7 @@ __device__ __noinline__ void run_gemm_tc(const Params& P, const Stage& st, char*
     }
     const GemmMember& M = (mi == pf) ? ctrl_of(smem)->mem : P.members[st.mem0 + mi];
     if (mi != cur) {
+      __syncthreads();   // every warp is done with the previous member's program before it is replaced
       G = stage_prog(P, M.prog, cache_of(smem, 0));
       cur = mi;
     }

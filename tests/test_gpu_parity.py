@@ -238,3 +238,28 @@ def test_bert_pattern_repeated_launches_reuse_workspace():
     for o in outs:
         assert float(np.abs(o - emu).max()) <= 2e-2
     assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[1], outs[2])
+
+
+@pytest.mark.parametrize("flags", [L.FLAG_NO_PATTERN, L.FLAG_NO_PATTERN | L.FLAG_NO_GLOBAL_SYNC])
+def test_lstm_generic_fused_executor(flags):
+    """The generic fused executor on a stacked LSTM with hidden 256: horizontally fused GEMV groups of
+    several members (warp-per-output skinny-GEMM path, member switches inside a CTA's task loop)."""
+    cfg = dict(synth.LSTM_CFG, steps=12, layers=4, hidden=256, input=256, w_dtype="f32")
+    gt, wt, gs, ws, plan = _lstm_case(cfg, flags, reps=2)
+    assert "GEMM_SIMT" in plan.describe()
+    assert rel_err(gt, wt) <= 1e-4
+    assert rel_err(gs, ws) <= 1e-4
+
+
+@pytest.mark.parametrize("flags", [L.FLAG_NO_PATTERN, L.FLAG_NO_PATTERN | L.FLAG_NO_VERTICAL | L.FLAG_NO_GLOBAL_SYNC])
+def test_bert_base_generic_fused_executor(flags):
+    """BERT-base (2 layers) on the generic fused executor (the Table 4 V1 / V3 rungs)."""
+    cfg = dict(synth.BERT_BASE, layers=2)
+    x = synth.bert_input(cfg)
+    w = synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    emu = te.evaluate(spec, og.bert_feed(X, plist, x, w), bf16_operands=True)[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    (out,), plan = run(g, og.bert_feed(gX, gpl, x, w), [gy], flags)
+    assert "not used" in plan.describe().splitlines()[0]
+    assert float(np.abs(out - emu).max()) <= 2e-2
