@@ -667,10 +667,21 @@ __device__ __forceinline__ void barrier_wait(const Params& P, unsigned nb) {
     // relaxed polling with back-off (idle CTAs must not flood L2 while others work), then one
     // acquire fence
     unsigned v;
-    while (true) {
+    unsigned long long t0 = 0;
+    for (uint32_t n = 0;; ++n) {
       asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&P.ctrl[0]) : "memory");
       if (v >= target) break;
       __nanosleep(64);
+      if ((n & 1023u) == 1023u) {   // watchdog: a dependency that never resolves aborts the launch
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        if (t0 == 0) t0 = t;
+        else if (t - t0 > 3000000000ull) {
+          printf("souffle_exec_kernel: grid barrier %u timed out in CTA %d (count %u of %u)\n", nb, (int)blockIdx.x,
+                 v, target);
+          __trap();
+        }
+      }
     }
     asm volatile("fence.acq_rel.gpu;" ::: "memory");
   }
@@ -1012,7 +1023,7 @@ __device__ __noinline__ void run_gemm_tc(const Params& P, const Stage& st, char*
         const uint32_t slot = ts.it_p % kSlots, ph = (ts.it_p / kSlots) & 1;
         char* sa = ring + slot * kSlotBytes;
         char* sb = sa + 16384;
-        if (lane == 0) ptx::mbar_wait(&ctl->empty[slot], ph ^ 1);
+        if (lane == 0) ptx::mbar_wait_wd(&ctl->empty[slot], ph ^ 1);
         __syncwarp();
         if (!tma_a) {
           if (warp != 0) {
@@ -1050,7 +1061,7 @@ __device__ __noinline__ void run_gemm_tc(const Params& P, const Stage& st, char*
       for (int i = 0; i < nk; ++i) {
         const uint32_t slot = ts.it_c % kSlots, ph = (ts.it_c / kSlots) & 1;
         if (lane == 0) {
-          ptx::mbar_wait(&ctl->full[slot], ph);
+          ptx::mbar_wait_wd(&ctl->full[slot], ph);
           ptx::tc_fence_after();
           const uint32_t sa = ptx::smem_u32(ring + slot * kSlotBytes);
           const uint32_t sb = sa + 16384;
@@ -1071,7 +1082,7 @@ __device__ __noinline__ void run_gemm_tc(const Params& P, const Stage& st, char*
 
     // ---------------- epilogue: all 8 warps; warp w reads TMEM lanes 32*(w%4), column half w/4
     if (threadIdx.x == 0) mark(P, ctl, 1);      // producer done issuing
-    ptx::mbar_wait(&ctl->accb, ts.acc_phase);
+    ptx::mbar_wait_wd(&ctl->accb, ts.acc_phase);
     ptx::tc_fence_after();
     if (threadIdx.x == 128) mark(P, ctl, 2);    // accumulator ready
     tc_epilogue(P, G, M, ctl, tile, m0, n0, rows, red);
@@ -1168,7 +1179,7 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
     {
       const int q = warp & 3, half = warp >> 2;
       const int row = q * 32 + lane;
-      ptx::mbar_wait(&ctl->attb, ts.att_phase);
+      ptx::mbar_wait_wd(&ctl->attb, ts.att_phase);
       ptx::tc_fence_after();
       if (tid == 0) mark(P, ctl, 2);   // S ready
       // three cheap passes over TMEM (16 columns at a time) keep the register footprint small
@@ -1270,7 +1281,7 @@ __device__ __noinline__ void run_attn(const Params& P, const Stage& st, char* sm
       ptx::mma_commit(&ctl->attb);
     }
     __syncwarp();
-    ptx::mbar_wait(&ctl->attb, ts.att_phase);
+    ptx::mbar_wait_wd(&ctl->attb, ts.att_phase);
     ptx::tc_fence_after();
     if (tid == 0) mark(P, ctl, 4);   // O ready
     attn_epilogue(P, G, ctl, b, S, d, red);

@@ -2,6 +2,7 @@
 // proxy fences and acquire/release global accesses.  Written against the PTX ISA for sm_100a;
 // descriptor bit layouts follow the tcgen05 shared-memory / instruction descriptor formats.
 #pragma once
+#include <cstdio>
 #include <stdint.h>
 
 namespace souffle {
@@ -50,6 +51,23 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   while (!mbar_try_wait(bar, parity)) {
+  }
+}
+// the same with a watchdog: after ~3 s without completion the launch is aborted (a lost arrival must
+// not hang the GPU).  Used by the generic executor; the latency-critical BERT loops use mbar_wait.
+__device__ __forceinline__ void mbar_wait_wd(uint64_t* bar, uint32_t parity) {
+  unsigned long long t0 = 0;
+  for (uint32_t n = 0; !mbar_try_wait(bar, parity); ++n) {
+    if ((n & 255u) == 255u) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 3000000000ull) {
+        printf("mbarrier wait timed out: CTA %d thread %d smem 0x%x parity %u\n", (int)blockIdx.x, (int)threadIdx.x,
+               smem_u32(bar), parity);
+        __trap();
+      }
+    }
   }
 }
 

@@ -55,7 +55,24 @@ def test_swin_tiny_bf16_tensor_cores():
     assert np.max(np.abs(again - ref)) <= 2e-2
 
 
-def test_swin_b_batch1_full_size():
+def _swin_b_child():
     got, again, ref, plan = _run(S.SWIN_B, bf16=True)
-    assert got.shape == (1, 1000)
-    assert np.max(np.abs(got - ref)) <= 2e-2, np.max(np.abs(got - ref))
+    print("RESULT", got.shape[0], got.shape[1], float(np.max(np.abs(got - ref))), float(np.max(np.abs(again - ref))))
+
+
+def test_swin_b_batch1_full_size():
+    """Full Swin-B at batch 1 against the bf16-operand oracle.  Runs in a fresh process: after the BERT
+    kernel has run in the same process, a later Swin-B launch can stall (known issue, DESIGN.md §9;
+    the executor's watchdog turns the stall into a launch error instead of a hung GPU)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_swin as t; t._swin_b_child()" % (
+        root, os.path.join(root, "tests"))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, cwd=root)
+    line = [ln for ln in r.stdout.splitlines() if ln.startswith("RESULT")]
+    assert line, r.stderr[-2000:]
+    _, b, n, e1, e2 = line[0].split()
+    assert (int(b), int(n)) == (1, 1000)
+    assert float(e1) <= 2e-2 and float(e2) <= 2e-2, (e1, e2)
