@@ -136,6 +136,7 @@ struct Params {
   int32_t n_stages_total;
   int32_t n_zero;
   int32_t first, count, cooperative, uses_tc, is_last;
+  unsigned int* progress;     // per-CTA (stage << 8 | point) of thread 0, read by the watchdog
   void* bufs[MAX_BUFS];
 };
 

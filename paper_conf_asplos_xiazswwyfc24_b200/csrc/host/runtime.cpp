@@ -35,7 +35,8 @@ size_t workspace_bytes(Plan& p) {
   w.ctrl_off = 0;
   // barrier words + stage timestamps + 8 sub-stage marks per stage
   w.ctrl_bytes = al(256 + 8 * ((int64_t)p.stages.size() + 1) + 64 * (int64_t)p.stages.size() +
-                        (p.profiling ? 8 * 4 * 160 * (int64_t)p.stages.size() : 0), 256);
+                        (p.profiling ? 8 * 4 * 160 * (int64_t)p.stages.size() : 0), 256) +
+                 1024;   // + per-CTA progress words (watchdog diagnostics)
   int64_t o = w.ctrl_bytes;
   w.prog_off = o;
   int64_t q = 0;
@@ -204,6 +205,7 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
   prm.ws_data = base + w.data_off;
   prm.ctrl = (unsigned int*)(base + w.ctrl_off);
   prm.prof = p.profiling ? (unsigned long long*)(base + w.ctrl_off + 256) : nullptr;
+  prm.progress = (unsigned int*)(base + w.ctrl_off + w.ctrl_bytes - 1024);
   prm.n_stages_total = (int32_t)p.stages.size();
   for (size_t i = 0; i < p.buf_ptr.size(); ++i) prm.bufs[i] = p.buf_ptr[i];
   cudaStream_t s = (cudaStream_t)stream;

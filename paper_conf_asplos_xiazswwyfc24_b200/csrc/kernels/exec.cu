@@ -642,6 +642,10 @@ __device__ __forceinline__ void flush_reds(const Params& P, const Prog& G, int64
   for (int k = 0; k < MAX_RED; ++k) red[k] = 0.f;
 }
 
+__device__ __forceinline__ void progress(const Params& P, int stage, int point) {
+  if (threadIdx.x == 0 && blockIdx.x < 256) *(volatile unsigned*)&P.progress[blockIdx.x] = ((unsigned)stage << 8) | (unsigned)point;
+}
+
 // ================================================================== grid barrier
 // Split-phase barrier on a monotonically increasing counter.  arrive: all threads order their
 // global writes (generic proxy) before the async proxy (TMA) of other CTAs, the CTA synchronises,
@@ -679,6 +683,11 @@ __device__ __forceinline__ void barrier_wait(const Params& P, unsigned nb) {
         else if (t - t0 > 3000000000ull) {
           printf("souffle_exec_kernel: grid barrier %u timed out in CTA %d (count %u of %u)\n", nb, (int)blockIdx.x,
                  v, target);
+          const unsigned mine = *(volatile unsigned*)&P.progress[blockIdx.x];
+          for (int c = 0; c < (int)gridDim.x && c < 256; ++c) {
+            const unsigned pc = *(volatile unsigned*)&P.progress[c];
+            if ((pc >> 8) < (mine >> 8)) printf("  lagging CTA %d: stage %u point %u\n", c, pc >> 8, pc & 255u);
+          }
           __trap();
         }
       }
@@ -1082,12 +1091,16 @@ __device__ __noinline__ void run_gemm_tc(const Params& P, const Stage& st, char*
 
     // ---------------- epilogue: all 8 warps; warp w reads TMEM lanes 32*(w%4), column half w/4
     if (threadIdx.x == 0) mark(P, ctl, 1);      // producer done issuing
+    progress(P, ctl->cur_stage, 1);
     ptx::mbar_wait_wd(&ctl->accb, ts.acc_phase);
     ptx::tc_fence_after();
     if (threadIdx.x == 128) mark(P, ctl, 2);    // accumulator ready
+    progress(P, ctl->cur_stage, 2);
     tc_epilogue(P, G, M, ctl, tile, m0, n0, rows, red);
+    progress(P, ctl->cur_stage, 3);
     ts.acc_phase ^= 1;
     __syncthreads();
+    progress(P, ctl->cur_stage, 4);
   }
   if (threadIdx.x == 0) ctl->ts = ts;
   __syncthreads();
@@ -1328,8 +1341,13 @@ __global__ void __launch_bounds__(kThreads, 1) souffle_exec_kernel(const __grid_
         P.prof[P.n_stages_total + 1 + 8 * s + 6] = (unsigned long long)clock64();   // SM clock at start
       }
     }
+    progress(P, s, 0);
     __syncthreads();
     const Stage& st = *sst;
+    // read before the stage's closing __syncthreads: once a thread is past it, prefetch_stage may
+    // overwrite the staged descriptor with stage s+1's, and a lagging warp would then take s+1's
+    // barrier decision (a mismatched barrier sequence that stalled one CTA forever)
+    const bool bar = P.cooperative && st.barrier_after;
     switch (st.kind) {
       case ST_EW: run_ew(P, st, smem); break;
       case ST_REDUCE: run_reduce(P, st, smem); break;
@@ -1340,7 +1358,7 @@ __global__ void __launch_bounds__(kThreads, 1) souffle_exec_kernel(const __grid_
     __syncthreads();
     if (s + 1 < P.first + P.count) {
       // split-phase barrier: arrive, prefetch the next stage's static data, then wait
-      const bool bar = P.cooperative && st.barrier_after;
+      progress(P, s, 9);
       if (bar) barrier_arrive(P, nb, ctl);
       prefetch_stage(P, s + 1, smem);
       if (bar) barrier_wait(P, nb);
