@@ -388,7 +388,7 @@ def main():
                          "stages": mplan.exec_info()["stages"]}
         del msess, mplan
         # Swin-B runs in a child process (fresh CUDA context) with a time limit: a launch that trips a
-        # kernel watchdog must not take the whole bench line with it (known issue)
+        # kernel watchdog must not take the whole bench line with it
         progress("Swin-B (child process)")
         import subprocess as sp
         try:

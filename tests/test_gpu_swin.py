@@ -61,9 +61,8 @@ def _swin_b_child():
 
 
 def test_swin_b_batch1_full_size():
-    """Full Swin-B at batch 1 against the bf16-operand oracle.  Runs in a fresh process: after the BERT
-    kernel has run in the same process, a later Swin-B launch can stall (known issue, DESIGN.md §9;
-    the executor's watchdog turns the stall into a launch error instead of a hung GPU)."""
+    """Full Swin-B at batch 1 against the bf16-operand oracle, in a fresh process (isolated from the
+    kernels the other tests ran; this is how a stall fixed this round was first contained)."""
     import os
     import subprocess
     import sys
