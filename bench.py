@@ -310,7 +310,9 @@ def main():
     dev = torch.device(f"cuda:{local}")
     stream = torch.cuda.current_stream(dev)
     progress("building BERT-base plan")
+    t_plan = time.perf_counter()
     g, plan, sess, X, y, x_host = build_bert(local)
+    t_plan = time.perf_counter() - t_plan
     progress("timing BERT-base")
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
     launches_per_step = plan.exec_info()["launches"]
@@ -424,7 +426,8 @@ def main():
             "config": {"workload": WORKLOAD, "l2": "256 MB flush before every timed step (outside the events)",
                        "parallelism": f"replicas x{ws} (batch-sharded, no collective on the hot path)",
                        "kernels_per_inference": info["launches"], "stages": info["stages"],
-                       "grid_barriers": info["barriers"]},
+                       "grid_barriers": info["barriers"],
+                       "plan_and_bind_s": round(t_plan, 2)},   # analysis + partition + lowering + bind (host)
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s", "frac": achieved / hbm,
                          "traffic": traffic, "peak_source": src,
                          "algorithmic_bytes_per_launch": ALGO_BYTES,
