@@ -385,9 +385,29 @@ def main():
         progress("MMoE")
         mplan, msess = build_mmoe(local)
         tm = time_steps(msess, 50, 3, flush, stream)
+        # a single event-bracketed launch of a ~5 us kernel is dominated by launch overhead; also time
+        # 100 back-to-back inferences in one bracket, and an empty kernel in the same bracket as context
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(100):
+            msess.run()
+        b.record(stream)
+        b.synchronize()
+        dummy = torch.zeros(1, device=dev)
+        td = []
+        for i in range(30):
+            c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            c0.record(stream)
+            dummy.add_(1)
+            c1.record(stream)
+            c1.synchronize()
+            if i >= 5:
+                td.append(c0.elapsed_time(c1) * 1e3)
         extra["mmoe"] = {"workload": "MMoE 8 experts x 16, 2 tasks, d_in 100, batch 1 (fp32)",
                          "latency_us": statistics.median(tm) * 1e3, "launches": mplan.exec_info()["launches"],
-                         "stages": mplan.exec_info()["stages"]}
+                         "stages": mplan.exec_info()["stages"],
+                         "back_to_back_us_per_inference": a.elapsed_time(b) * 1e3 / 100,
+                         "empty_kernel_same_bracket_us": statistics.median(td)}
         del msess, mplan
         # Swin-B runs in a child process (fresh CUDA context) with a time limit: a launch that trips a
         # kernel watchdog must not take the whole bench line with it
