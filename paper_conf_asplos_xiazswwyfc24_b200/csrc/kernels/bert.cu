@@ -94,21 +94,23 @@ __device__ __forceinline__ void spin_guard(uint32_t& n, unsigned long long& t0) 
 }
 
 // ------------------------------------------------------------------ grid barrier (split phase)
-__device__ __forceinline__ void grid_arrive(const BertParams& P, int k) {
-  ptx::fence_proxy_async();   // generic-proxy writes of this stage -> TMA reads of later stages
+__device__ __forceinline__ void grid_arrive(const BertParams& P, int k, bool tma_consumed) {
+  // generic-proxy writes of this stage -> TMA reads of later stages (split-K partials are read by
+  // plain loads of the LayerNorm rows: no proxy fence for those stages)
+  if (tma_consumed) ptx::fence_proxy_async();
   csync();
   if (threadIdx.x == 0) {
     __threadfence();
     atomicAdd(&P.ctrl[k], 1u);
   }
 }
-__device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target_arrivals) {
+__device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target_arrivals, bool tma_reads) {
   if (threadIdx.x == 0) {
     const unsigned target = (unsigned)target_arrivals;
     uint32_t n = 0;
     unsigned long long t0 = 0;
     while (ptx::ld_acquire(&P.ctrl[k]) < target) spin_guard(n, t0);
-    ptx::fence_proxy_async();
+    if (tma_reads) ptx::fence_proxy_async();   // the stage reads other CTAs' data through TMA
   }
   csync();
 }
@@ -643,7 +645,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
     const bool work = has_work(P, st);
     if (work && s > 0) {
       if (st.fwait) flag_wait(st, st.kind == BS_ATTN ? (int)blockIdx.x % st.heads : (int)blockIdx.x % st.nsplit);
-      else grid_wait(P, s - 1, prev_workers);
+      else grid_wait(P, s - 1, prev_workers, st.kind != BS_ROW);
     }
     prev_workers = st.workers;
     if (s + 1 < P.nstages && tid < (int)(sizeof(BStage) / 16))
@@ -670,7 +672,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
         }
       }
       if (tid == 0) submark(P, st, 6);
-      if (st.arrive) grid_arrive(P, s);
+      if (st.arrive) grid_arrive(P, s, st.kind == BS_ROW || (st.kind == BS_GEMM && st.epi != EP_PARTIAL));
       if (tid == 0) submark(P, st, 7);
     }
     csync();   // descriptor s+1 visible; everyone is done with descriptor s
