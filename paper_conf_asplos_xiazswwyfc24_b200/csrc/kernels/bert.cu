@@ -648,8 +648,12 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
       else grid_wait(P, s - 1, prev_workers, st.kind != BS_ROW);
     }
     prev_workers = st.workers;
-    if (s + 1 < P.nstages && tid < (int)(sizeof(BStage) / 16))
-      reinterpret_cast<int4*>(sbuf + ((s + 1) & 1))[tid] = __ldg(reinterpret_cast<const int4*>(P.stages + s + 1) + tid);
+    // stage s+1's descriptor is copied by warp 7 (an epilogue-only warp in GEMM stages): thread 0 issues
+    // the stage's first TMA / MMA and must not stall on this L2 load
+    constexpr int kDescWarp = 7 * 32, kDescVecs = (int)(sizeof(BStage) / 16);
+    if (s + 1 < P.nstages && tid >= kDescWarp && tid < kDescWarp + kDescVecs)
+      reinterpret_cast<int4*>(sbuf + ((s + 1) & 1))[tid - kDescWarp] =
+          __ldg(reinterpret_cast<const int4*>(P.stages + s + 1) + (tid - kDescWarp));
     if (tid == 0) {
       mark(P, s);
       C->cur_stage = s;
