@@ -278,6 +278,21 @@ def swin_child(dev_index):
                       "lowering": "generic fused-subprogram executor (exec.cu)"}))
 
 
+def relaunch_under_torchrun(n):
+    """`python bench.py --gpus N` without a launcher: re-exec under torch.distributed.run with one
+    rank per GPU (127.0.0.1 rendezvous), so N really means N replicas and the max over ranks."""
+    import socket
+    so = socket.socket()
+    so.bind(("127.0.0.1", 0))
+    port = so.getsockname()[1]
+    so.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    progress("re-executing under torchrun: " + " ".join(cmd[1:]))
+    sys.stdout.flush()
+    os.execv(sys.executable, cmd)
+
+
 def progress(msg):
     print(f"[bench {time.strftime('%H:%M:%S')}] {msg}", file=sys.stderr, flush=True)
 
@@ -301,9 +316,13 @@ def main():
         run_reference(args)
         return
 
+    ws, rank, local = dist_env()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        relaunch_under_torchrun(args.gpus)          # does not return
+    if ws != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}: launch one rank per GPU")
     import torch
     import torch.distributed as dist
-    ws, rank, local = dist_env()
     if ws > 1:
         dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
     torch.cuda.set_device(local)
@@ -331,7 +350,7 @@ def main():
     value = R.aggregate_rate(args.steps, total_ms / 1e3)  # inferences of all ranks / max time
     # after timing: gather every replica's output to rank 0 over NCCL (the only collective) and check
     # the replicas agree (same request -> same result; the oracle check itself is in tests/)
-    gathered = R.gather_to_rank0(sess.outputs[y])
+    gathered = R.gather_to_rank0(sess.outputs[y].unsqueeze(0))
     replica_check = None
     if gathered is not None:
         replica_check = {"replicas": int(gathered.shape[0]),

@@ -193,8 +193,9 @@ souffle_status souffle_bind(souffle_plan p, souffle_tensor t, void* device_ptr);
  * reusable state afterwards (barrier counters are reset by the last CTA to leave). */
 souffle_status souffle_workspace_init(souffle_plan p, void* workspace, void* stream);
 /* Enqueue the whole program on `stream`: one cooperative launch per subprogram (or one launch
- * per TE under SOUFFLE_FLAG_UNFUSED).  Asynchronous; never allocates or synchronises.  A plan may
- * run concurrently on different streams only with distinct workspaces. */
+ * per TE under SOUFFLE_FLAG_UNFUSED).  Asynchronous; never allocates or synchronises.  A plan is
+ * tied to the ONE workspace last passed to souffle_workspace_init (E_STATE for any other): to run
+ * a model concurrently on several streams, create one plan (and workspace) per stream. */
 souffle_status souffle_run(souffle_plan p, void* workspace, void* stream);
 
 /* ------------------------------------------------------------------ debug profiling
@@ -202,7 +203,9 @@ souffle_status souffle_run(souffle_plan p, void* workspace, void* stream);
  * barrier) and the last CTA records the launch end, in the workspace control region.
  * souffle_plan_read_profile synchronises the device and returns one duration (microseconds) per
  * stage in execution order: time from the stage's start to the next stage's start (so it
- * includes the grid barrier that follows the stage).  Debug use only (it synchronises). */
+ * includes the grid barrier that follows the stage).  Debug use only (it synchronises).
+ * Changing the flag changes the workspace layout: call it BEFORE souffle_plan_workspace_bytes /
+ * souffle_workspace_init (otherwise souffle_run returns E_STATE until they are called again). */
 souffle_status souffle_plan_set_profiling(souffle_plan p, int32_t on);
 souffle_status souffle_plan_read_profile(souffle_plan p, void* workspace, double* stage_us, int32_t cap,
                                          int32_t* n);
@@ -210,6 +213,15 @@ souffle_status souffle_plan_read_profile(souffle_plan p, void* workspace, double
  * per stage (stage-kind specific, 0 if unused).  cap >= 9 * stages + 1. */
 souffle_status souffle_plan_read_profile_raw(souffle_plan p, void* workspace, uint64_t* stamps, int32_t cap,
                                              int32_t* n);
+
+/* Test introspection of the BERT pattern kernel (kernels/bert.cu, host/bert.cpp): byte offset from
+ * the workspace base and size of one of its named activation buffers -- "xb" / "l1b" (bf16 [S][H]
+ * GEMM A operands), "l1f" / "xf" (fp32 [S][H] residual stream), "qk" (bf16 Q then K, head-major
+ * [2*heads][S][64]), "vt" (bf16 V^T [heads][64][S]), "h" (bf16 GELU output [S][F]), "part_o" /
+ * "part_2" (fp32 split-K partials [nsplit][S][H]).  Used with SOUFFLE_BERT_STAGES=b,e (run only
+ * stages [b, e)) by the stage-isolation tests.  Errors: E_INVALID_ARG (unknown name, NULL
+ * pointers), E_UNSUPPORTED (the plan does not use the BERT pattern kernel). */
+souffle_status souffle_plan_debug_region(souffle_plan p, const char* name, int64_t* offset, int64_t* bytes);
 
 #ifdef __cplusplus
 }

@@ -317,5 +317,16 @@ def _add_raw_profile():
 
 _SIGS["souffle_plan_read_profile_raw"] = [C.c_void_p, C.c_void_p, C.POINTER(C.c_uint64), C.c_int32,
                                           C.POINTER(C.c_int32)]
+_SIGS["souffle_plan_debug_region"] = [C.c_void_p, C.c_char_p, C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
+
+
+def _debug_region(self, name):
+    """(byte offset, bytes) of a named BERT-kernel workspace buffer (stage-isolation tests)."""
+    o, b = C.c_int64(), C.c_int64()
+    check(self.lib.souffle_plan_debug_region(self.h, name.encode(), C.byref(o), C.byref(b)))
+    return o.value, b.value
+
+
+Plan.debug_region = _debug_region
 EXPORTS = sorted(list(_SIGS) + ["souffle_last_error", "souffle_version"])
 _add_raw_profile()

@@ -10,8 +10,11 @@
 //           EP_GELU    + bias, erf-GELU, bf16 [S][N]
 //           EP_PARTIAL split-K partial, fp32 [split][S][N] plain stores (summed by the consumer)
 //   ATTN  per head: QK^T -> scale -> max-subtracted softmax -> PV, S and O in TMEM (Fig. 1(c))
-//   ROW   per token row: sum of split-K partials + bias + residual + LayerNorm (two-pass mean /
-//         variance over the row), fp32 and bf16 outputs (the two-phase reduction of P:L527-536)
+//   ROW   per token row: sum of split-K partials + bias + residual + LayerNorm ((mean, M2) merged
+//         pairwise from exactly centred per-thread values, so a constant row gives beta), fp32 and bf16
+//         outputs (the two-phase reduction of P:L527-536).  Stage 0 (row_mode 0) converts the fp32
+//         input to bf16 and, on all CTAs, refreshes the packed constant vectors from the bound
+//         pointers.
 // Weights never depend on activations, so a producer warp streams every GEMM stage's weight tiles
 // through a shared-memory ring ahead of the grid barriers (§6.5 "cross-stage prefetch").
 #pragma once
@@ -67,6 +70,14 @@ struct alignas(16) BStage {
   uint16_t* r_out_b;
 };
 
+// one constant vector (bias / gamma / beta) refreshed from its bound pointer into the packed
+// workspace copy by stage 0 of every launch (so an in-place update of a bound parameter is seen)
+struct alignas(16) BCopy {
+  const float* src;
+  float* dst;
+  int32_t n, first;             // first: flat index of element 0 in the concatenation of all vectors
+};
+
 struct BertParams {
   const BStage* stages;
   const void* tmaps;            // CUtensorMap[] (128 B each)
@@ -76,6 +87,9 @@ struct BertParams {
   int32_t nstages, S;
   int32_t dbg_skip;             // debug: bit k set -> stages of kind k do no work (barriers only)
   int32_t nflags;
+  const BCopy* copies;          // constant vectors refreshed in stage 0 (all CTAs take part)
+  int32_t ncopies, copy_total;  // entries, total floats
+  int32_t s_begin, s_end;       // stages executed: [0, nstages) except in stage-isolation tests
 };
 
 }  // namespace souffle

@@ -437,6 +437,27 @@ souffle_status souffle_plan_hgroup(souffle_plan p, souffle_tensor te, int32_t* l
     if (kind) *kind = gid >= 0 ? P.an.hkind[gid] : -1;
   });
 }
+souffle_status souffle_plan_debug_region(souffle_plan p, const char* name, int64_t* offset, int64_t* bytes) {
+  return guard([&] {
+    Plan& P = PL(p);
+    if (!name || !offset || !bytes) throw Error(SOUFFLE_E_INVALID_ARG, "null argument");
+    const BertPlan& b = P.bert;
+    if (!b.on) throw Error(SOUFFLE_E_UNSUPPORTED, "the plan does not use the BERT pattern kernel");
+    const int64_t S = b.S, H = b.H, F = b.F;
+    const std::string n(name);
+    if (n == "xb") { *offset = b.o_xb; *bytes = S * H * 2; }
+    else if (n == "l1b") { *offset = b.o_l1b; *bytes = S * H * 2; }
+    else if (n == "l1f") { *offset = b.o_l1f; *bytes = S * H * 4; }
+    else if (n == "xf") { *offset = b.o_xf; *bytes = S * H * 4; }
+    else if (n == "qk") { *offset = b.o_qk; *bytes = 2 * S * H * 2; }
+    else if (n == "vt") { *offset = b.o_vt; *bytes = S * H * 2; }
+    else if (n == "h") { *offset = b.o_h; *bytes = S * F * 2; }
+    else if (n == "part_o") { *offset = b.o_part_o; *bytes = (int64_t)b.out.nsplit * S * H * 4; }
+    else if (n == "part_2") { *offset = b.o_part_2; *bytes = (int64_t)b.ffn2.nsplit * S * H * 4; }
+    else throw Error(SOUFFLE_E_INVALID_ARG, "unknown debug region " + n);
+  });
+}
+
 souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t* stages, int32_t* barriers) {
   return guard([&] {
     Plan& P = PL(p);
@@ -502,7 +523,13 @@ souffle_status souffle_run(souffle_plan p, void* workspace, void* stream) {
 }
 
 souffle_status souffle_plan_set_profiling(souffle_plan p, int32_t on) {
-  return guard([&] { PL(p).profiling = on != 0; });
+  // the control region's size depends on the flag (runtime.cpp workspace_bytes): a change requires
+  // souffle_plan_workspace_bytes + souffle_workspace_init again, so mark the plan dirty
+  return guard([&] {
+    Plan& P = PL(p);
+    if (P.profiling != (on != 0)) P.dirty = true;
+    P.profiling = on != 0;
+  });
 }
 souffle_status souffle_plan_read_profile(souffle_plan p, void* workspace, double* stage_us, int32_t cap, int32_t* n) {
   g_err.clear();

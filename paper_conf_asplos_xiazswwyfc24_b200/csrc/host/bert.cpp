@@ -146,7 +146,10 @@ BertGemmCfg full_cfg(int64_t N, int64_t K, int sms, int max_nt, const char* env)
   }
   if (const char* e = std::getenv(env)) {
     int nt = 0;
-    if (std::sscanf(e, "%d", &nt) == 1 && nt > 0 && nt <= max_nt && N % nt == 0 && N / nt <= sms)
+    // the kernel's epilogues exist for n tiles of 16, 32, 64 and 128 only (max_nt: QKV tiles must not
+    // straddle a 64-wide head)
+    if (std::sscanf(e, "%d", &nt) == 1 && (nt == 16 || nt == 32 || nt == 64 || nt == 128) && nt <= max_nt &&
+        N % nt == 0 && N / nt <= sms)
       c = BertGemmCfg{nt, 1, (int)(K / 64), (int)(N / nt)};
   }
   return c;
@@ -173,7 +176,8 @@ BertGemmCfg split_cfg(int64_t N, int64_t K, int sms, const char* env) {
   }
   if (const char* e = std::getenv(env)) {   // SOUFFLE_BERT_<STAGE>=nt,kchunks
     int nt = 0, kch = 0;
-    if (std::sscanf(e, "%d,%d", &nt, &kch) == 2 && nt > 0 && N % nt == 0 && kch >= 1 && nt <= 128) {
+    if (std::sscanf(e, "%d,%d", &nt, &kch) == 2 && (nt == 16 || nt == 32 || nt == 64 || nt == 128) && N % nt == 0 &&
+        kch >= 1) {
       const int nsplit = (kc + kch - 1) / kch;
       if ((int64_t)(N / nt) * nsplit <= sms && nsplit <= 12) best = BertGemmCfg{nt, nsplit, kch, (int)(N / nt)};
     }
@@ -236,7 +240,7 @@ void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   bp.num_sms = dev.num_sms > 0 ? dev.num_sms : 148;
   const int sms = bp.num_sms;
   if (bp.S % 8) return no("S must be a multiple of 8 (V^T rows are TMA-loaded)");
-  if (bp.H > 768) return no("hidden size must be <= 768 (LayerNorm row stage: 3 columns per thread)");
+  if (bp.H > 768) return no("hidden size must be <= 768 (at most 12 heads of 64: split-K partials per LayerNorm row)");
   bp.qkv = full_cfg(3LL * bp.H, bp.H, sms, 64, "SOUFFLE_BERT_QKV");     // tiles never straddle a head
   // out-projection fused into attention: split-K over heads (K = 64 per head), N tiles of nt rows
   bp.out = BertGemmCfg{};
@@ -270,6 +274,7 @@ void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   // all small per-layer vectors packed contiguously (a handful of 2 MB pages instead of ~200
   // scattered allocations: every TLB miss is a microsecond on the critical path)
   bp.o_consts = take((int64_t)bp.layers.size() * (9 * H + F) * 4);
+  bp.o_copies = take((int64_t)bp.layers.size() * 10 * (int64_t)sizeof(BCopy));
   bp.total = al(o, 4096);
   bp.on = true;
 }
@@ -459,8 +464,10 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
   if ((int)st.size() != bp.nstages) return fail(SOUFFLE_E_STATE, "internal: stage count");
   for (int i = 0; i < (int)st.size(); ++i) {
     st[i].idx = i;
-    // barrier arrivals = CTAs with work (must match has_work() in kernels/bert.cu)
-    st[i].workers = st[i].kind == BS_ROW ? std::min(bp.S, bp.num_sms) : st[i].ntasks;
+    // barrier arrivals = CTAs with work (must match has_work() in kernels/bert.cu); stage 0 (convert +
+    // constant refresh) runs on every CTA
+    st[i].workers = st[i].kind == BS_ROW ? (st[i].row_mode == 0 ? bp.num_sms : std::min(bp.S, bp.num_sms))
+                                         : st[i].ntasks;
   }
   for (int i = 0; i + 1 < (int)st.size(); ++i) st[i].arrive = st[i + 1].fwait ? 0 : 1;
   cudaStream_t s = (cudaStream_t)stream;
@@ -468,9 +475,22 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(base + bp.o_stages, st.data(), st.size() * sizeof(BStage), cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = cudaMemcpyAsync(base + bp.o_tmaps, tm.data(), tm.size(), cudaMemcpyHostToDevice, s);
-  for (size_t i = 0; i < packed.size() && e == cudaSuccess; ++i)
-    e = cudaMemcpyAsync(base + packed[i].second, ptr(packed[i].first), 4 * numel(p.g.nodes[packed[i].first].shape),
-                        cudaMemcpyDeviceToDevice, s);
+  // constant vectors: copied from the bound pointers by stage 0 of every launch (BCopy table)
+  std::vector<BCopy> cp;
+  int total = 0;
+  for (auto& q : packed) {
+    BCopy c;
+    c.src = (const float*)ptr(q.first);
+    c.dst = (float*)(base + q.second);
+    c.n = (int)numel(p.g.nodes[q.first].shape);
+    c.first = total;
+    total += c.n;
+    cp.push_back(c);
+  }
+  bp.ncopies = (int)cp.size();
+  bp.copy_total = total;
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(base + bp.o_copies, cp.data(), cp.size() * sizeof(BCopy), cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);   // host staging vectors die with this call
   if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("bert workspace init: ") + cudaGetErrorString(e));
   p.inited_ws = ws;
@@ -507,7 +527,21 @@ souffle_status bert_run(Plan& p, void* ws, void* stream) {
   prm.nstages = bp.nstages;
   prm.nflags = bp.nflags;
   prm.S = bp.S;
+  prm.copies = (const BCopy*)(base + bp.o_copies);
+  prm.ncopies = bp.ncopies;
+  prm.copy_total = bp.copy_total;
   if (const char* dbg = std::getenv("SOUFFLE_BERT_DBG_SKIP")) prm.dbg_skip = std::atoi(dbg);   // timing studies
+  prm.s_begin = 0;
+  prm.s_end = bp.nstages;
+  // stage-isolation tests (tests/test_gpu_bert_stages.py): run only stages [b, e) on a workspace the
+  // test pre-filled (the integer bit-exact checks of single GEMM stages)
+  if (const char* se = std::getenv("SOUFFLE_BERT_STAGES")) {
+    int b = 0, en = 0;
+    if (std::sscanf(se, "%d,%d", &b, &en) == 2 && 0 <= b && b < en && en <= bp.nstages) {
+      prm.s_begin = b;
+      prm.s_end = en;
+    }
+  }
   cudaError_t e = bert_launch(prm, grid, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("bert launch: ") + cudaGetErrorString(e));
   return SOUFFLE_OK;

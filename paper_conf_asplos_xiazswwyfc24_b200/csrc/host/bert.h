@@ -39,8 +39,10 @@ struct BertPlan {
   int64_t o_ctrl = 0, o_stages = 0, o_tmaps = 0, o_prof = 0;
   int64_t o_xb = 0, o_ctx = 0, o_l1b = 0, o_l1f = 0, o_xf = 0;
   int64_t o_h = 0, o_qk = 0, o_vt = 0, o_part_o = 0, o_part_2 = 0;
-  int64_t o_consts = 0;          // packed per-layer fp32 vectors (bias / gamma / beta), snapshot at init
+  int64_t o_consts = 0;          // packed per-layer fp32 vectors (bias / gamma / beta), refreshed by stage 0
+  int64_t o_copies = 0;          // BCopy table: bound vector -> packed copy
   int64_t total = 0;
+  int ncopies = 0, copy_total = 0;   // constant-refresh table (set at workspace init)
 };
 
 // Fills bp (bp.on = true) if g is a BERT encoder stack that the specialised kernel implements.

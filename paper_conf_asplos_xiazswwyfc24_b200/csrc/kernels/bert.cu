@@ -6,19 +6,22 @@
 // (§6.4 "global sync", Fig. 2):
 //
 //   warp 8      weight producer: walks the stage list and TMA-loads, for every GEMM task this CTA
-//               owns, its weight K-chunks into an 8 x 16 KB shared-memory ring.  Weights are
+//               owns, its weight K-chunks into a BW_SLOTS x 16 KB shared-memory ring.  Weights are
 //               constants, so it runs ahead across grid barriers and the HBM weight stream overlaps
 //               the activation dependency chain (§6.5 cross-stage prefetch, Table 4 V4).
 //   warps 0-7   stage executor:
-//     GEMM      A (bf16 activations) streamed by TMA through a 5-slot ring; one thread issues
+//     GEMM      A (bf16 activations) streamed by TMA through a BA_SLOTS-slot ring; one thread issues
 //               tcgen05.mma (M = 128 tokens, N = tile, K = 16) into TMEM; fused epilogues:
 //               bias + bf16 + head-major / transposed stores (QKV: the reshape/permute index maps
-//               of §6.2 folded into the store), bias + erf-GELU (FFN1), or fp32 split-K partials.
+//               of §6.2 folded into the store), bias + erf-GELU (FFN1), or fp32 split-K partials;
+//               stored straight from registers (every thread owns >= 16 contiguous bytes of a
+//               token row, or a 64-byte coalesced run of V^T), the bias loaded during the mainloop.
 //     ATTN      per head: Q, K, V^T by TMA, S = QK^T in TMEM, softmax (max-subtracted, fp32
 //               registers), P bf16 in smem, O = PV in TMEM, ctx stored bf16 (Fig. 1(c), §2.3).
 //     ROW       one CTA per token row: sum of the split-K partials + bias + residual, LayerNorm
-//               with two-pass block reductions, fp32 and bf16 outputs (two-phase reduction,
-//               partial results per block, combined after the global sync).
+//               with (mean, M2) statistics merged pairwise (one block reduction), fp32
+//               and bf16 outputs (two-phase reduction: partial results per block,
+//               combined after the global sync).
 //   A split-phase grid barrier (one arrival counter per barrier) separates dependent stages.
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -142,7 +145,7 @@ __device__ __forceinline__ void flag_wait(const BStage& st, int idx) {
 __device__ __forceinline__ bool has_work(const BertParams& P, const BStage& st) {
   const int b = blockIdx.x;
   if (st.kind == BS_GEMM || st.kind == BS_ATTN) return b < st.ntasks;
-  return b < P.S;
+  return st.row_mode == 0 || b < P.S;   // stage 0 (convert + constant refresh) runs on every CTA
 }
 
 // K-chunk order of a task: rotated by the CTA index so that the CTAs of a stage, which all read
@@ -161,7 +164,7 @@ __device__ __forceinline__ int wgroup(int nt) { return max(1, BW_SLOT_BYTES / (n
 __device__ void weight_producer(const BertParams& P, Ctrl* C, char* wring) {
   const char* tmaps = (const char*)P.tmaps;
   uint32_t it = 0;
-  for (int s = 0; s < P.nstages; ++s) {
+  for (int s = P.s_begin; s < P.s_end; ++s) {
     const BStage* st = P.stages + s;
     const int kind = __ldg(&st->kind);
     if (kind != BS_GEMM && kind != BS_ATTN) continue;   // ATTN: fused out-projection tile
@@ -197,83 +200,96 @@ struct MmaState {
   uint32_t accph, attph, qkvph;
 };
 
-// Epilogue of one 128 x nt accumulator tile: TMEM -> registers (+bias, GELU) -> fp32 staging tile in
-// shared memory (the A region, free once the MMAs completed) -> coalesced full-sector global stores
-// by the whole CTA (thread-per-row stores would write 16-byte fragments of 128 different lines).
+// Epilogue of one 128 x nt accumulator tile, straight from registers: warp w reads TMEM lanes
+// 32*(w%4).. (token rows) and column half w/4, adds the bias it loaded while the MMAs ran
+// (bias_half: COLS fp32 values of this thread's half, 16-byte aligned), and stores its row segment:
+// fp32 partial (COLS*4 B), bf16 GELU / Q / K (COLS*2 B >= 16 B) or V^T (one bf16 per feature row;
+// the 32 lanes of a warp write 64 contiguous bytes).  Rows >= S (TMA zero-fill) are not stored.
 template <int COLS>
-__device__ __forceinline__ void gemm_epilogue(const BertParams& P, const BStage& st, Ctrl* C, char* stage_smem, int n0,
-                                              int split) {
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int q = warp & 3, half = warp >> 2;
-  const int row = q * 32 + lane;
-  const int S = P.S, N = st.N;
-  constexpr int NT = 2 * COLS;
-  constexpr int LD = NT + 4;   // padded fp32 row stride of the staging tile
-  float* stg = reinterpret_cast<float*>(stage_smem);
-  const uint32_t taddr = C->tmem_base + ((uint32_t)(q * 32) << 16) + half * COLS;
-  float v[COLS];
+__device__ __forceinline__ void tmem_row(Ctrl* C, float* v) {
+  const int warp = threadIdx.x >> 5;
+  const uint32_t taddr = C->tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + (warp >> 2) * COLS;
   if constexpr (COLS == 8) ptx::tmem_ld8(taddr, v);
   else if constexpr (COLS == 16) ptx::tmem_ld16(taddr, v);
   else if constexpr (COLS == 32) ptx::tmem_ld32(taddr, v);
   else ptx::tmem_ld64(taddr, v);
   ptx::tc_fence_before();
-  if (st.epi != EP_PARTIAL) {
-    const float4* bp = reinterpret_cast<const float4*>(st.bias + n0 + half * COLS);
+}
+
+// fp32 split-K partial [split][S][N] (out-projection per head, FFN2 per K range): no bias
+template <int COLS>
+__device__ __forceinline__ void tail_partial(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0,
+                                             int split) {
+  ptx::mbar_wait(&C->accb, ms.accph);
+  ms.accph ^= 1;
+  ptx::tc_fence_after();
+  if (threadIdx.x == 0) submark(P, st, 3);
+  float v[COLS];
+  tmem_row<COLS>(C, v);
+  const int warp = threadIdx.x >> 5, row = (warp & 3) * 32 + (threadIdx.x & 31);
+  if (row >= P.S) return;
+  float4* dst = reinterpret_cast<float4*>(st.part + ((int64_t)split * P.S + row) * st.N + n0 + (warp >> 2) * COLS);
 #pragma unroll
-    for (int c = 0; c < COLS; c += 4) {
-      const float4 b = __ldg(bp + c / 4);
-      v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
-    }
-    if (st.epi == EP_GELU) {
+  for (int c = 0; c < COLS; c += 4) dst[c / 4] = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+}
+
+// + bias, then erf-GELU -> bf16 [S][N] (FFN1), or bf16 Q / K head-major and V^T (QKV, the reshape /
+// permute index maps of §6.2 folded into the store).  Tiles of <= 32 columns load their bias while
+// the MMAs run (warps 2-7 are idle in the mainloop); wider tiles after the accumulator.
+template <int COLS>
+__device__ __forceinline__ void tail_bias(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0) {
+  const int warp = threadIdx.x >> 5, half = warp >> 2, row = (warp & 3) * 32 + (threadIdx.x & 31);
+  const int c0 = n0 + half * COLS;
+  constexpr bool kEarly = COLS <= 16;
+  float4 bq[kEarly ? COLS / 4 : 1];
+  if constexpr (kEarly) {
 #pragma unroll
-      for (int c = 0; c < COLS; ++c) v[c] = gelu_erf(v[c]);
-    }
+    for (int c = 0; c < COLS; c += 4) bq[c / 4] = __ldg(reinterpret_cast<const float4*>(st.bias + c0 + c));
   }
+  ptx::mbar_wait(&C->accb, ms.accph);
+  ms.accph ^= 1;
+  ptx::tc_fence_after();
+  if (threadIdx.x == 0) submark(P, st, 3);
+  float v[COLS];
+  tmem_row<COLS>(C, v);
+  if (row >= P.S) return;
 #pragma unroll
-  for (int c = 0; c < COLS; c += 4)
-    *reinterpret_cast<float4*>(stg + row * LD + half * COLS + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
-  csync();
-  if (st.epi == EP_PARTIAL) {
-    constexpr int U = NT / 4;   // float4 units per row
-    float* dst = st.part + (int64_t)split * S * N + n0;
-    for (int u = tid; u < S * U; u += BERT_COMPUTE) {
-      const int r = u / U, c4 = u % U;
-      *reinterpret_cast<float4*>(dst + (int64_t)r * N + 4 * c4) = *reinterpret_cast<const float4*>(stg + r * LD + 4 * c4);
-    }
-  } else if (st.epi == EP_GELU) {
-    constexpr int U = NT / 8;   // 8-element (16 B) bf16 units per row
-    uint16_t* dst = st.out_b + n0;
-    for (int u = tid; u < S * U; u += BERT_COMPUTE) {
-      const int r = u / U, c8 = u % U;
-      const float* sp = stg + r * LD + 8 * c8;
-      *reinterpret_cast<uint4*>(dst + (int64_t)r * N + 8 * c8) =
-          make_uint4(pack_bf16(sp[0], sp[1]), pack_bf16(sp[2], sp[3]), pack_bf16(sp[4], sp[5]), pack_bf16(sp[6], sp[7]));
-    }
-  } else {
-    // EP_QKV: columns [n0, n0 + NT) of [Q | K | V] lie in one head (NT divides 64)
-    const int H = N / 3;
-    const int which = n0 / H, hh = (n0 % H) >> 6, jd = n0 & 63;
-    if (which < 2) {   // head-major [S][64]: NT * 2 bytes contiguous per token row
-      constexpr int U = NT / 8;
-      uint16_t* dst = st.out_b + ((int64_t)(which * st.heads + hh) * S << 6) + jd;
-      for (int u = tid; u < S * U; u += BERT_COMPUTE) {
-        const int r = u / U, c8 = u % U;
-        const float* sp = stg + r * LD + 8 * c8;
-        *reinterpret_cast<uint4*>(dst + ((int64_t)r << 6) + 8 * c8) =
-            make_uint4(pack_bf16(sp[0], sp[1]), pack_bf16(sp[2], sp[3]), pack_bf16(sp[4], sp[5]), pack_bf16(sp[6], sp[7]));
-      }
-    } else {           // V^T [64][S]: S * 2 bytes contiguous per feature row
-      const int U = S / 8;
-      uint16_t* dst = st.out_vt + ((int64_t)hh * 64 + jd) * S;
-      for (int u = tid; u < NT * U; u += BERT_COMPUTE) {
-        const int dcol = u / U, t8 = u % U;
-        const float* sp = stg + (8 * t8) * LD + dcol;
-        *reinterpret_cast<uint4*>(dst + (int64_t)dcol * S + 8 * t8) =
-            make_uint4(pack_bf16(sp[0], sp[LD]), pack_bf16(sp[2 * LD], sp[3 * LD]), pack_bf16(sp[4 * LD], sp[5 * LD]),
-                       pack_bf16(sp[6 * LD], sp[7 * LD]));
-      }
-    }
+  for (int c = 0; c < COLS; c += 4) {
+    const float4 b = kEarly ? bq[kEarly ? c / 4 : 0] : __ldg(reinterpret_cast<const float4*>(st.bias + c0 + c));
+    v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
   }
+  const int S = P.S, N = st.N;
+  if (st.epi == EP_GELU) {
+#pragma unroll
+    for (int c = 0; c < COLS; ++c) v[c] = gelu_erf(v[c]);
+    uint4* dst = reinterpret_cast<uint4*>(st.out_b + (int64_t)row * N + c0);
+#pragma unroll
+    for (int c = 0; c < COLS; c += 8)
+      dst[c / 8] = make_uint4(pack_bf16(v[c], v[c + 1]), pack_bf16(v[c + 2], v[c + 3]), pack_bf16(v[c + 4], v[c + 5]),
+                              pack_bf16(v[c + 6], v[c + 7]));
+    return;
+  }
+  // EP_QKV: columns [n0, n0 + 2*COLS) of [Q | K | V] lie in one head (the tile width divides 64)
+  const int H = N / 3;
+  const int which = n0 / H, hh = (n0 % H) >> 6, jd = (n0 & 63) + half * COLS;
+  if (which < 2) {   // head-major [S][64]: COLS*2 contiguous bytes per token row
+    uint4* dst = reinterpret_cast<uint4*>(st.out_b + (((int64_t)(which * st.heads + hh) * S + row) << 6) + jd);
+#pragma unroll
+    for (int c = 0; c < COLS; c += 8)
+      dst[c / 8] = make_uint4(pack_bf16(v[c], v[c + 1]), pack_bf16(v[c + 2], v[c + 3]), pack_bf16(v[c + 4], v[c + 5]),
+                              pack_bf16(v[c + 6], v[c + 7]));
+  } else {           // V^T [64][S]: a warp writes 32 consecutive tokens (64 B) of one feature row
+    uint16_t* dst = st.out_vt + ((int64_t)hh * 64 + jd) * S + row;
+#pragma unroll
+    for (int c = 0; c < COLS; ++c) dst[(int64_t)c * S] = bf16_bits(v[c]);
+  }
+}
+
+template <int COLS>
+__device__ __forceinline__ void gemm_tail(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0,
+                                          int split) {
+  if (st.epi == EP_PARTIAL) tail_partial<COLS>(P, st, C, ms, n0, split);
+  else tail_bias<COLS>(P, st, C, ms, n0);
 }
 
 __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* wring, char* areg, MmaState& ms) {
@@ -336,15 +352,11 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
   }
 
   // ---- epilogue (all 8 warps: warp w reads TMEM lanes 32*(w%4).., column half w/4)
-  ptx::mbar_wait(&C->accb, ms.accph);
-  ms.accph ^= 1;
-  ptx::tc_fence_after();
-  if (tid == 0) submark(P, st, 3);
   switch (nt) {
-    case 16: gemm_epilogue<8>(P, st, C, areg, n0, split); break;
-    case 32: gemm_epilogue<16>(P, st, C, areg, n0, split); break;
-    case 64: gemm_epilogue<32>(P, st, C, areg, n0, split); break;
-    default: gemm_epilogue<64>(P, st, C, areg, n0, split); break;
+    case 16: gemm_tail<8>(P, st, C, ms, n0, split); break;
+    case 32: gemm_tail<16>(P, st, C, ms, n0, split); break;
+    case 64: gemm_tail<32>(P, st, C, ms, n0, split); break;
+    default: gemm_tail<64>(P, st, C, ms, n0, split); break;
   }
   if (tid == 0) submark(P, st, 4);
   if (st.fout) flag_signal(st, n0);
@@ -400,22 +412,24 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
     ptx::tc_fence_after();
     if (tid == 0) submark(P, st, 2);
     const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + half * 64;
-    const float scale = st.scale;
+    // p_j = 2^(s_j c - m c) / z with c = scale * log2(e): one FFMA + one MUFU.EX2 per score
+    const float c = st.scale * 1.4426950408889634f;
     float sv[64];
     ptx::tmem_ld64(tb, sv);
     float mx = -INFINITY;
 #pragma unroll
     for (int j = 0; j < 64; ++j) {
-      sv[j] = (half * 64 + j < S) ? sv[j] * scale : -INFINITY;
+      if (half * 64 + j >= S) sv[j] = -INFINITY;   // keys beyond S (TMA zero-fill)
       mx = fmaxf(mx, sv[j]);
     }
     // each half normalises with its own max; one (max, sum) exchange combines the halves:
-    // z = z_a e^{m_a - m} + z_b e^{m_b - m}, p_j = e^{s_j - m_a} e^{m_a - m} / z
-    float z = 0.f;
+    // z = z_a 2^{(m_a - m)c} + z_b 2^{(m_b - m)c}, p_j = 2^{(s_j - m_a)c} 2^{(m_a - m)c} / z
     const float mxs = (mx == -INFINITY) ? 0.f : mx;   // a fully masked half contributes 0
+    const float mc = mxs * c;
+    float z = 0.f;
 #pragma unroll
     for (int j = 0; j < 64; ++j) {
-      sv[j] = __expf(sv[j] - mxs);
+      sv[j] = ptx::ex2(fmaf(sv[j], c, -mc));
       z += sv[j];
     }
     float2* xch = reinterpret_cast<float2*>(Qs);   // [2][128] (max, sum); Q is consumed (S complete)
@@ -423,8 +437,9 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
     csync();
     const float2 o = xch[(half ^ 1) * 128 + row];
     const float m = fmaxf(mx, o.x);
-    const float zt = z * __expf(mxs - m) + (o.x == -INFINITY ? 0.f : o.y * __expf(o.x - m));
-    const float iz = __expf(mxs - m) / zt;   // p_j = sv[j] * iz
+    const float fa = ptx::ex2((mxs - m) * c);
+    const float zt = z * fa + (o.x == -INFINITY ? 0.f : o.y * ptx::ex2((o.x - m) * c));
+    const float iz = fa / zt;   // p_j = sv[j] * iz
 #pragma unroll
     for (int c0 = 0; c0 < 64; c0 += 8) {
       *reinterpret_cast<uint4*>(Ps + half * 16384 + sw128(row, c0 * 2)) =
@@ -481,99 +496,114 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
     __syncwarp();
     ++ms.wit;
   }
-  ptx::mbar_wait(&C->accb, ms.accph);
-  ms.accph ^= 1;
-  ptx::tc_fence_after();
   if (tid == 0) submark(P, st, 5);
-  // split index = head, N tile = jt
+  // split index = head, N tile = jt (EP_PARTIAL: no bias)
   switch (st.nt) {
-    case 16: gemm_epilogue<8>(P, st, C, areg, jt * st.nt, h); break;
-    case 32: gemm_epilogue<16>(P, st, C, areg, jt * st.nt, h); break;
-    case 64: gemm_epilogue<32>(P, st, C, areg, jt * st.nt, h); break;
-    default: gemm_epilogue<64>(P, st, C, areg, jt * st.nt, h); break;
+    case 16: tail_partial<8>(P, st, C, ms, jt * st.nt, h); break;
+    case 32: tail_partial<16>(P, st, C, ms, jt * st.nt, h); break;
+    case 64: tail_partial<32>(P, st, C, ms, jt * st.nt, h); break;
+    default: tail_partial<64>(P, st, C, ms, jt * st.nt, h); break;
   }
 }
 
 // ------------------------------------------------------------------ row stage (one CTA per row)
-// one fused block reduction of (sum v, sum v^2)
-__device__ __forceinline__ float2 block_sum2(Ctrl* C, float2 x) {
+// Row statistics by pairwise (Chan) merging of (mean, M2 = sum of squared deviations): every
+// thread centres its own 4 values exactly, equal-count merges in the warp tree, then the warps in
+// order.  A constant row gives mean = the value and M2 = 0 exactly (so LayerNorm outputs beta, as
+// the fp64 definition does), and an offset row (1e3 + noise) keeps the noise (no E[x^2] - E[x]^2
+// cancellation).  Active threads = whole warps (cols is a multiple of 128); returns (mean, M2).
+__device__ __forceinline__ float2 block_welford(Ctrl* C, float m, float M2, int nwarps) {
+  float n = 4.f;
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
-    x.x += __shfl_xor_sync(0xffffffffu, x.x, o);
-    x.y += __shfl_xor_sync(0xffffffffu, x.y, o);
+  for (int o = 1; o < 32; o <<= 1) {
+    const float mb = __shfl_xor_sync(0xffffffffu, m, o);
+    const float Mb = __shfl_xor_sync(0xffffffffu, M2, o);
+    const float dl = mb - m;
+    M2 = (M2 + Mb) + dl * dl * (0.5f * n);
+    m = (m + mb) * 0.5f;   // commutative: both lanes of a pair hold the identical value
+    n *= 2.f;
   }
-  if ((threadIdx.x & 31) == 0) {
-    C->red[0][threadIdx.x >> 5] = x.x;
-    C->red[1][threadIdx.x >> 5] = x.y;
+  const int w = threadIdx.x >> 5;
+  if ((threadIdx.x & 31) == 0 && w < nwarps) {
+    C->red[0][w] = m;
+    C->red[1][w] = M2;
   }
   csync();
-  float2 s = make_float2(0.f, 0.f);
-#pragma unroll
-  for (int w = 0; w < 8; ++w) {
-    s.x += C->red[0][w];
-    s.y += C->red[1][w];
+  float mean = C->red[0][0], q = C->red[1][0], na = 128.f;
+  for (int k = 1; k < nwarps; ++k) {
+    const float mb = C->red[0][k], dl = mb - mean;
+    const float nn = na + 128.f;
+    mean += dl * (128.f / nn);
+    q += C->red[1][k] + dl * dl * (na * 128.f / nn);
+    na = nn;
   }
-  return s;
+  return make_float2(mean, q);
 }
 
-constexpr int kRowPer = 3;   // columns per thread: cols <= 768
 constexpr int kMaxSplit = 12;   // split-K partials summed by a LayerNorm row
+// stage 0, all CTAs: refresh the packed constant vectors (bias / gamma / beta) from the bound
+// pointers, so the later stages (which read the packed copy: a few 2 MB pages instead of ~200
+// scattered allocations) always see the current parameter values
+__device__ void refresh_consts(const BertParams& P) {
+  const int G = gridDim.x * BERT_COMPUTE;
+  int e = 0;
+  for (int i = blockIdx.x * BERT_COMPUTE + threadIdx.x; i < P.copy_total; i += G) {
+    while (e + 1 < P.ncopies && __ldg(&P.copies[e + 1].first) <= i) ++e;
+    const BCopy* cp = P.copies + e;
+    const int k = i - __ldg(&cp->first);
+    float* dst = (float*)__ldg(reinterpret_cast<const unsigned long long*>(&cp->dst));
+    dst[k] = __ldg(reinterpret_cast<const float*>(ldgp(&cp->src)) + k);
+  }
+}
+
+// one CTA per token row; thread t < cols/4 owns columns 4t..4t+3 (cols <= 1024)
 __device__ void run_row(const BertParams& P, const BStage& st, Ctrl* C) {
   const int tid = threadIdx.x;
   const int S = P.S, cols = st.cols;
+  const bool mine = 4 * tid < cols;
   for (int r = blockIdx.x; r < S; r += gridDim.x) {
     if (st.row_mode == 0) {
-#pragma unroll
-      for (int i = 0; i < kRowPer; ++i) {
-        const int c = tid + 256 * i;
-        if (c < cols) st.r_out_b[(int64_t)r * cols + c] = bf16_bits(__ldg(st.r_in + (int64_t)r * cols + c));
+      if (mine) {
+        const float4 x = __ldg(reinterpret_cast<const float4*>(st.r_in + (int64_t)r * cols) + tid);
+        reinterpret_cast<uint2*>(st.r_out_b + (int64_t)r * cols)[tid] = make_uint2(pack_bf16(x.x, x.y), pack_bf16(x.z, x.w));
       }
       continue;
     }
-    // sum of the split-K partials + bias + residual, with gamma / beta: every load of the row is
-    // issued before any is used (one L2 round trip)
-    float v[kRowPer], g[kRowPer], be[kRowPer];
-    float t[kMaxSplit][kRowPer];
+    // sum of the split-K partials + bias + residual: every load of the row is issued before any is
+    // used (one L2 round trip)
     const int ns = st.r_nsplit;
     const float* part = st.r_in + (int64_t)r * cols;
     const int64_t pstride = (int64_t)S * cols;
+    float4 v = make_float4(0.f, 0.f, 0.f, 0.f), g = v, be = v;
+    float m = 0.f, M2 = 0.f;
+    if (mine) {
+      const float4 b = __ldg(reinterpret_cast<const float4*>(st.r_bias) + tid);
+      const float4 x = __ldcg(reinterpret_cast<const float4*>(st.r_res + (int64_t)r * cols) + tid);
+      float4 t[kMaxSplit];
 #pragma unroll
-    for (int i = 0; i < kRowPer; ++i) {
-      const int c = tid + 256 * i;
-      const bool in = c < cols;
-      v[i] = in ? __ldg(st.r_bias + c) + __ldcg(st.r_res + (int64_t)r * cols + c) : 0.f;
-      g[i] = in ? __ldg(st.r_gamma + c) : 0.f;
-      be[i] = in ? __ldg(st.r_beta + c) : 0.f;
+      for (int u = 0; u < kMaxSplit; ++u)
+        t[u] = u < ns ? __ldcg(reinterpret_cast<const float4*>(part + u * pstride) + tid) : make_float4(0.f, 0.f, 0.f, 0.f);
+      g = __ldg(reinterpret_cast<const float4*>(st.r_gamma) + tid);
+      be = __ldg(reinterpret_cast<const float4*>(st.r_beta) + tid);
+      float4 a = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-      for (int u = 0; u < kMaxSplit; ++u) t[u][i] = (u < ns && in) ? __ldcg(part + u * pstride + c) : 0.f;
-    }
-#pragma unroll
-    for (int i = 0; i < kRowPer; ++i) {
-      float a = 0.f;
-#pragma unroll
-      for (int u = 0; u < kMaxSplit; ++u) a += t[u][i];
-      v[i] += a;
+      for (int u = 0; u < kMaxSplit; ++u) { a.x += t[u].x; a.y += t[u].y; a.z += t[u].z; a.w += t[u].w; }
+      v = make_float4((b.x + x.x) + a.x, (b.y + x.y) + a.y, (b.z + x.z) + a.z, (b.w + x.w) + a.w);
+      m = ((v.x + v.y) + (v.z + v.w)) * 0.25f;
+      const float d0 = v.x - m, d1 = v.y - m, d2 = v.z - m, d3 = v.w - m;
+      M2 = (d0 * d0 + d1 * d1) + (d2 * d2 + d3 * d3);
     }
     if (tid == 0) submark(P, st, 0);
-    float2 sq = make_float2(0.f, 0.f);
-#pragma unroll
-    for (int i = 0; i < kRowPer; ++i) {   // out-of-range columns hold 0
-      sq.x += v[i];
-      sq.y += v[i] * v[i];
-    }
-    sq = block_sum2(C, sq);   // one-pass statistics (R10): one barrier instead of two
-    const float mu = sq.x / (float)cols;
-    const float var = fmaxf(sq.y / (float)cols - mu * mu, 0.f);
+    const float2 mq = block_welford(C, m, M2, cols >> 7);   // one block reduction (R10)
+    const float mu = mq.x, var = mq.y / (float)cols;
     const float rs = rsqrtf(var + st.eps);
     if (tid == 0) submark(P, st, 1);
-#pragma unroll
-    for (int i = 0; i < kRowPer; ++i) {
-      const int c = tid + 256 * i;
-      if (c < cols) {
-        const float o = (v[i] - mu) * rs * g[i] + be[i];
-        if (st.r_out_f) st.r_out_f[(int64_t)r * cols + c] = o;
-        if (st.r_out_b) st.r_out_b[(int64_t)r * cols + c] = bf16_bits(o);
-      }
+    if (mine) {
+      const float4 o = make_float4((v.x - mu) * rs * g.x + be.x, (v.y - mu) * rs * g.y + be.y,
+                                   (v.z - mu) * rs * g.z + be.z, (v.w - mu) * rs * g.w + be.w);
+      if (st.r_out_f) reinterpret_cast<float4*>(st.r_out_f + (int64_t)r * cols)[tid] = o;
+      if (st.r_out_b)
+        reinterpret_cast<uint2*>(st.r_out_b + (int64_t)r * cols)[tid] = make_uint2(pack_bf16(o.x, o.y), pack_bf16(o.z, o.w));
     }
     csync();   // C->red is reused by the next row of this CTA
   }
@@ -611,39 +641,25 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
   if (warp == 8) {
     const int lane = tid & 31;
     if (lane == 0) weight_producer(P, C, wring);   // ---- weight producer
-    if (lane == 1) {
-      // ---- warm L2 with the stage table and every stage's small constant vectors
-      if (blockIdx.x == 0) ptx::prefetch_l2(P.stages, (uint32_t)(P.nstages * sizeof(BStage)));
-      for (int s = blockIdx.x; s < P.nstages; s += gridDim.x) {
-        const BStage* sp = P.stages + s;
-        const int kind = __ldg(&sp->kind);
-        if (kind == BS_ROW && __ldg(&sp->row_mode) == 1) {
-          const uint32_t b = 4u * __ldg(&sp->cols);
-          ptx::prefetch_l2(ldgp(&sp->r_bias), b);
-          ptx::prefetch_l2(ldgp(&sp->r_gamma), b);
-          ptx::prefetch_l2(ldgp(&sp->r_beta), b);
-        } else if (kind == BS_GEMM && __ldg(&sp->epi) != EP_PARTIAL) {
-          ptx::prefetch_l2(ldgp(&sp->bias), 4u * __ldg(&sp->N));
-        }
-      }
-    }
+    if (lane == 1 && blockIdx.x == 0) ptx::prefetch_l2(P.stages, (uint32_t)(P.nstages * sizeof(BStage)));   // stage table
     return;
   }
   // ---- stage executor (warps 0-7).  Stage descriptors are double-buffered in smem: stage s+1's is
   // fetched while stage s runs, so it is never on the critical path behind a grid barrier.
   MmaState ms{0u, 0u, 0u, 0u, 0u, 0u};
   if (tid < (int)(sizeof(BStage) / 16))
-    reinterpret_cast<int4*>(sbuf)[tid] = __ldg(reinterpret_cast<const int4*>(P.stages) + tid);
+    reinterpret_cast<int4*>(sbuf + (P.s_begin & 1))[tid] = __ldg(reinterpret_cast<const int4*>(P.stages + P.s_begin) + tid);
   csync();
   // Barrier participation: only the CTAs with work in stage s arrive at barrier s (its target is
   // st.workers), and a CTA waits for barrier s-1 only before a stage it works in.  Ordering stays
   // transitive because every stage has at least one worker, and each worker waited for the
   // previous barrier before its own arrival.
   int prev_workers = 0;
-  for (int s = 0; s < P.nstages; ++s) {
+  // [s_begin, s_end) is the whole stage list except in the stage-isolation tests (debug)
+  for (int s = P.s_begin; s < P.s_end; ++s) {
     const BStage& st = sbuf[s & 1];
     const bool work = has_work(P, st);
-    if (work && s > 0) {
+    if (work && s > P.s_begin) {
       if (st.fwait) flag_wait(st, st.kind == BS_ATTN ? (int)blockIdx.x % st.heads : (int)blockIdx.x % st.nsplit);
       else grid_wait(P, s - 1, prev_workers, st.kind != BS_ROW);
     }
@@ -651,7 +667,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
     // stage s+1's descriptor is copied by warp 7 (an epilogue-only warp in GEMM stages): thread 0 issues
     // the stage's first TMA / MMA and must not stall on this L2 load
     constexpr int kDescWarp = 7 * 32, kDescVecs = (int)(sizeof(BStage) / 16);
-    if (s + 1 < P.nstages && tid >= kDescWarp && tid < kDescWarp + kDescVecs)
+    if (s + 1 < P.s_end && tid >= kDescWarp && tid < kDescWarp + kDescVecs)
       reinterpret_cast<int4*>(sbuf + ((s + 1) & 1))[tid - kDescWarp] =
           __ldg(reinterpret_cast<const int4*>(P.stages + s + 1) + (tid - kDescWarp));
     if (tid == 0) {
@@ -663,7 +679,10 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
         switch (st.kind) {
           case BS_GEMM: run_gemm(P, st, C, wring, areg, ms); break;
           case BS_ATTN: run_attn(P, st, C, wring, areg, ms); break;
-          default: run_row(P, st, C); break;
+          default:
+            if (st.row_mode == 0) refresh_consts(P);
+            run_row(P, st, C);
+            break;
         }
       } else if ((st.kind == BS_GEMM || st.kind == BS_ATTN) && tid == 0) {
         // keep the weight ring in step with the producer: consume (and release) this task's groups

@@ -42,10 +42,22 @@ def aggregate_rate(units_per_rank: int, max_seconds: float) -> float:
 
 
 def gather_to_rank0(t: torch.Tensor):
-    """Stack every rank's output tensor on rank 0 (for the parity check after timing); None elsewhere."""
+    """Every rank's output (shape [n_r, ...], n_r may differ by rank: uneven request shards) on
+    rank 0 as ONE tensor [sum n_r, ...] in rank order (for the parity check after timing); None
+    elsewhere.  Shards are padded to the largest n_r for the collective and trimmed afterwards."""
     ws, rank = world()
     if ws == 1:
-        return t.unsqueeze(0)
-    parts = [torch.empty_like(t) for _ in range(ws)]
-    dist.all_gather(parts, t.contiguous())
-    return torch.stack(parts) if rank == 0 else None
+        return t
+    dev = t.device
+    n = torch.tensor([t.shape[0]], dtype=torch.int64, device=dev)
+    ns = [torch.zeros_like(n) for _ in range(ws)]
+    dist.all_gather(ns, n)
+    sizes = [int(x.item()) for x in ns]
+    mx = max(sizes)
+    pad = torch.zeros((mx,) + tuple(t.shape[1:]), dtype=t.dtype, device=dev)
+    pad[: t.shape[0]] = t
+    parts = [torch.empty_like(pad) for _ in range(ws)]
+    dist.all_gather(parts, pad)
+    if rank != 0:
+        return None
+    return torch.cat([p[:k] for p, k in zip(parts, sizes)])

@@ -195,3 +195,18 @@ def test_swin_graph_matches_oracle_builder_and_analysis():
                 ref = an.index_map(spec, t, s)
                 if ref is not None:
                     assert plan.index_map(t, s, int(np.prod(shapes[t]))) == ref, (t, s)
+
+
+def test_library_bfs_order_and_reuse_kind_goldens():
+    """The C library reproduces the hand-derived goldens (not only the oracle): Kahn-FIFO order
+    (tests/golden/bfs_order.json) and spatial vs temporal reuse (tests/golden/reuse_spatial.json)."""
+    import json
+    from test_oracle_analysis import _golden_bfs_spec, _qkv_spec
+    spec, gold = _golden_bfs_spec()
+    plan = M.from_spec(spec).partition(L.device_b200())
+    assert plan.bfs_order() == gold["order"]
+    for chain, kind in ((False, 0), (True, 1)):
+        spec, ids = _qkv_spec(chain)
+        plan = M.from_spec(spec).partition(L.device_b200())
+        cs, k = plan.reuse_set(ids["X"])
+        assert k == kind and cs == an.reuse_sets(spec)[ids["X"]][0]

@@ -27,7 +27,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, ws, port, q):
+def _worker(rank, ws, port, q, n_req):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=ws)
@@ -37,28 +37,32 @@ def _worker(rank, ws, port, q):
         t = R.max_over_ranks(1.0 + rank)
         rate = R.aggregate_rate(10, t)
         # each rank's replica output = its shard of request ids, gathered on rank 0 for checking
-        mine = torch.tensor([float(i) for i in R.shard(6, ws, rank)])
+        mine = torch.tensor([[float(i), 10.0 * i] for i in R.shard(n_req, ws, rank)]).reshape(-1, 2)
         got = R.gather_to_rank0(mine)
         if rank == 0:
-            q.put((t, rate, got.reshape(-1).tolist()))
+            q.put((t, rate, got[:, 0].tolist(), got[:, 1].tolist()))
         else:
             assert got is None
     finally:
         dist.destroy_process_group()
 
 
-@pytest.mark.timeout(120)
-def test_gloo_world_size_2():
+@pytest.mark.timeout(180)
+@pytest.mark.parametrize("ws,n_req", [(2, 6), (3, 7), (3, 2)])
+def test_gloo_replicas(ws, n_req):
+    """world_size 2 with equal shards, 3 ranks x 7 requests (shards 3/2/2) and 3 ranks x 2 requests
+    (one rank has an EMPTY shard): max-over-ranks time, aggregate rate, ordered gather."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    ps = [ctx.Process(target=_worker, args=(r, ws, port, q, n_req)) for r in range(ws)]
     for p in ps:
         p.start()
     for p in ps:
-        p.join(100)
+        p.join(150)
         assert p.exitcode == 0
-    t, rate, ids = q.get(timeout=10)
-    assert t == 2.0                      # max over ranks
-    assert rate == 2 * 10 / 2.0          # units of all ranks / slowest time
-    assert ids == [0, 1, 2, 3, 4, 5]     # shards gathered in rank order cover the stream once
+    t, rate, ids, tens = q.get(timeout=10)
+    assert t == float(ws)                    # max over ranks (rank r "took" 1 + r)
+    assert rate == ws * 10 / float(ws)       # units of all ranks / slowest time
+    assert ids == [float(i) for i in range(n_req)]   # shards gathered in rank order cover the stream once
+    assert tens == [10.0 * i for i in range(n_req)]

@@ -1,0 +1,9 @@
+#!/bin/bash
+# round-2 GPU call: parity of the BERT kernel, stage timeline, short bench (no extras)
+mkdir -p gpurun_out
+python -c "from paper_conf_asplos_xiazswwyfc24_b200.build import build; build()" > gpurun_out/build.log 2>&1
+timeout 900 python -m pytest tests/test_gpu_bert_stages.py tests/test_gpu_parity.py -q -x -m gpu -k "bert or stage or layernorm or bias" > gpurun_out/pytest_bert.txt 2>&1
+echo "pytest rc=$?" >> gpurun_out/pytest_bert.txt
+timeout 300 python tools/profile_bert.py 12 > gpurun_out/timeline.txt 2>&1
+timeout 600 python bench.py --steps 50 --warmup 5 --no-cpu-baseline --no-v0 --no-models > gpurun_out/bench_quick.json 2> gpurun_out/bench_quick.err
+echo done
