@@ -261,21 +261,27 @@ def time_steps(sess, steps, warmup, flush, stream, clk=None):
 
 
 def swin_child(dev_index):
-    """Swin-B b1 latency (the `swin` extra of the bench line), printed as one JSON object."""
+    """Swin-B (BASELINE.json configs[4]) through the Swin pattern kernels: batch-1 latency and
+    images/s at per-GPU batch 8 and 64 (the batch-sharded replica size of 64 images on 1 GPU), with
+    the tensor-pipe fraction; printed as one JSON object (the `swin` extra of the bench line)."""
     import torch
     torch.cuda.set_device(dev_index)
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=f"cuda:{dev_index}")
-    splan, ssess, scfg = build_swin(dev_index)
-    ts = time_steps(ssess, 10, 3, flush, stream)
-    _, tf, _ = peaks()
-    slat = statistics.median(ts) * 1e3
-    si = splan.exec_info()
-    print(json.dumps({"workload": "Swin-B 224x224 (torchvision swin_b), batch 1 per GPU (bf16 GEMM operands)",
-                      "latency_us": slat, "images_per_s": 1e6 / slat, "launches": si["launches"],
-                      "stages": si["stages"], "grid_barriers": si["barriers"],
-                      "tensor_frac": SWIN_FLOPS / (slat * 1e-6) / 1e12 / tf,
-                      "lowering": "generic fused-subprogram executor (exec.cu)"}))
+    _, tf, src = peaks()
+    out = {"workload": "Swin-B 224x224 (torchvision swin_b semantics), bf16 GEMM operands, fp32 elsewhere",
+           "flops_per_image": SWIN_FLOPS, "peak_tflops": tf, "peak_source": src}
+    for batch in (1, 8, 64):
+        splan, ssess, scfg = build_swin(dev_index, batch=batch)
+        ts = time_steps(ssess, 10 if batch < 64 else 5, 3, flush, stream)
+        lat = statistics.median(ts) * 1e3
+        si = splan.exec_info()
+        out[f"b{batch}"] = {"latency_us": lat, "images_per_s": batch * 1e6 / lat, "launches": si["launches"],
+                            "tensor_frac": SWIN_FLOPS * batch / (lat * 1e-6) / 1e12 / tf}
+        del ssess, splan
+    out["lowering"] = "pattern swin (kernels/swin.cu: tcgen05 GEMMs with fused epilogues, window attention, " \
+                      "LN gathers) replayed as one CUDA graph"
+    print(json.dumps(out))
 
 
 def relaunch_under_torchrun(n):

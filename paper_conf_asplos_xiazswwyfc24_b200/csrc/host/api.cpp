@@ -479,6 +479,12 @@ souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t
       if (barriers) *barriers = P.bert.nstages - 1;
       return;
     }
+    if (P.swin.on) {   // one kernel per fused subprogram, replayed as one CUDA graph
+      if (launches) *launches = P.swin.launches;
+      if (stages) *stages = P.swin.launches;
+      if (barriers) *barriers = 0;
+      return;
+    }
     if (launches) *launches = (int32_t)P.launches.size();
     if (stages) *stages = (int32_t)P.stages.size();
     if (barriers) *barriers = P.n_barriers;

@@ -192,7 +192,7 @@ enum { MAP_XB = 0, MAP_CTX = 1, MAP_L1B = 2, MAP_H = 3, MAP_QK = 4, MAP_VT = 5, 
 
 }  // namespace
 
-void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, BertPlan& bp) {
+void bert_match(const Graph& g, const Analysis& an, const souffle_device_desc& dev, uint32_t flags, BertPlan& bp) {
   bp = BertPlan();
   auto no = [&](const char* why) { bp.on = false; bp.why_not = why; };
   if (flags != 0) return no("ablation flags select the generic executor");
@@ -235,6 +235,21 @@ void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   }
   if (!c.ok || bp.layers.empty()) return no("TE program is not a BERT encoder stack");
   if (g.outputs.size() != 1 || g.outputs[0] != x) return no("the only output must be the last layer's LayerNorm");
+  // driven by the partition: one subprogram (one persistent launch), and per layer the QKV GEMM is the
+  // analysis' N-concat horizontal group of the three matmuls that read the layer input
+  if (an.num_sp != 1) return no("the partition has more than one subprogram");
+  for (size_t i = 0; i < g.nodes.size(); ++i)
+    if (g.nodes[i].op != SOUFFLE_OP_PLACEHOLDER && an.assign[i] != 0) return no("TE outside subprogram 0");
+  for (const BertLayerIds& L : bp.layers) {
+    int mm[3], k = 0;
+    for (size_t i = 0; i < g.nodes.size() && k < 3; ++i)
+      if (g.nodes[i].op == SOUFFLE_OP_MATMUL && (g.nodes[i].b == L.Wq || g.nodes[i].b == L.Wk || g.nodes[i].b == L.Wv))
+        mm[k++] = (int)i;
+    if (k != 3) return no("QKV matmuls");
+    const int gid = an.hgid[mm[0]];
+    if (gid < 0 || an.hgid[mm[1]] != gid || an.hgid[mm[2]] != gid || an.hkind[gid] != 0)
+      return no("the analysis did not group Q, K, V into one N-concat horizontal GEMM (§6.1)");
+  }
   bp.eps = eps;
   bp.Y = x;
   bp.num_sms = dev.num_sms > 0 ? dev.num_sms : 148;

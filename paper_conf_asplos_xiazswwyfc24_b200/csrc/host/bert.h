@@ -46,7 +46,10 @@ struct BertPlan {
 };
 
 // Fills bp (bp.on = true) if g is a BERT encoder stack that the specialised kernel implements.
-void bert_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, BertPlan& bp);
+// The match is driven by the partition (§5.4 / §6.1): the kernel runs ONE subprogram, so the
+// analysis must have put every TE into subprogram 0, and the [Q | K | V] horizontal GEMM is taken from
+// the analysis' horizontal group of the three matmuls (N-concat, shared A operand).
+void bert_match(const Graph& g, const Analysis& an, const souffle_device_desc& dev, uint32_t flags, BertPlan& bp);
 std::string bert_describe(const BertPlan& bp);
 
 }  // namespace souffle

@@ -8,6 +8,7 @@
 #include "bert.h"
 #include "lstm.h"
 #include "mmoe.h"
+#include "swin.h"
 #include "ir.h"
 
 namespace souffle {
@@ -60,6 +61,8 @@ struct Plan {
   BertPlan bert;                    // pattern lowering (bert.on: kernels/bert.cu runs the program)
   LstmPlan lstm;                    // pattern lowering (lstm.on: kernels/lstm.cu runs the program)
   MmoePlan mmoe;                    // pattern lowering (mmoe.on: kernels/mmoe.cu runs the program)
+  SwinPlan swin;                    // pattern lowering (swin.on: kernels/swin.cu, one CUDA graph)
+  ~Plan();
 };
 
 void lower(Plan& p);              // fills the lowered program + layout (pure host)

@@ -26,11 +26,14 @@ souffle_status bert_run(Plan& p, void* ws, void* stream);
 souffle_status lstm_init(Plan& p, void* ws, void* stream);
 souffle_status lstm_run(Plan& p, void* ws, void* stream);
 souffle_status mmoe_run(Plan& p, void* ws, void* stream);
+souffle_status swin_init(Plan& p, void* ws, void* stream);
+souffle_status swin_run(Plan& p, void* ws, void* stream);
 
 size_t workspace_bytes(Plan& p) {
   if (p.bert.on) return (size_t)p.bert.total;
   if (p.lstm.on) return (size_t)p.lstm.total;
   if (p.mmoe.on) return 256;
+  if (p.swin.on) return (size_t)p.swin.total;
   WsLayout& w = p.ws;
   w.ctrl_off = 0;
   // barrier words + stage timestamps + 8 sub-stage marks per stage
@@ -103,6 +106,7 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
     if (!p.buf_ptr[s]) return fail(SOUFFLE_E_STATE, "tensor " + std::to_string(p.buf_node[s]) + " is not bound");
   if (p.bert.on) return bert_init(p, ws, stream);
   if (p.lstm.on) return lstm_init(p, ws, stream);
+  if (p.swin.on) return swin_init(p, ws, stream);
   if (p.mmoe.on) {
     p.inited_ws = ws;
     p.dirty = false;
@@ -177,6 +181,11 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
     std::string why;
     if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
     return mmoe_run(p, ws, stream);
+  }
+  if (p.swin.on) {
+    std::string why;
+    if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
+    return swin_run(p, ws, stream);
   }
   static int max_active = -1;
   if (max_active < 0) {

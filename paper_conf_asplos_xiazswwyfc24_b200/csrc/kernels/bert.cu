@@ -216,21 +216,36 @@ __device__ __forceinline__ void tmem_row(Ctrl* C, float* v) {
   ptx::tc_fence_before();
 }
 
-// fp32 split-K partial [split][S][N] (out-projection per head, FFN2 per K range): no bias
+// fp32 split-K partial [split][S][N] (out-projection per head, FFN2 per K range): no bias.  Staged
+// through shared memory (the A region: its MMAs have completed) so every warp store instruction
+// writes 512 contiguous bytes -- thread-per-row float4 stores touch 32 lines per instruction and
+// measured 2x slower for these 32 KB tiles.  mk: debug mark index.
 template <int COLS>
 __device__ __forceinline__ void tail_partial(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0,
-                                             int split) {
+                                             int split, char* stage_smem, int mk) {
   ptx::mbar_wait(&C->accb, ms.accph);
   ms.accph ^= 1;
   ptx::tc_fence_after();
-  if (threadIdx.x == 0) submark(P, st, 3);
+  if (threadIdx.x == 0) submark(P, st, mk);
   float v[COLS];
   tmem_row<COLS>(C, v);
-  const int warp = threadIdx.x >> 5, row = (warp & 3) * 32 + (threadIdx.x & 31);
-  if (row >= P.S) return;
-  float4* dst = reinterpret_cast<float4*>(st.part + ((int64_t)split * P.S + row) * st.N + n0 + (warp >> 2) * COLS);
+  const int tid = threadIdx.x, warp = tid >> 5, half = warp >> 2, row = (warp & 3) * 32 + (tid & 31);
+  constexpr int NT = 2 * COLS, LD = NT + 4;   // padded fp32 row stride of the staging tile
+  float* stg = reinterpret_cast<float*>(stage_smem);
 #pragma unroll
-  for (int c = 0; c < COLS; c += 4) dst[c / 4] = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+  for (int c = 0; c < COLS; c += 4)
+    *reinterpret_cast<float4*>(stg + row * LD + half * COLS + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+  csync();
+  constexpr int U = NT / 4;   // float4 units per row
+  const int S = P.S, N = st.N;
+  float* dst = st.part + (int64_t)split * S * N + n0;
+  for (int u = tid; u < S * U; u += BERT_COMPUTE) {
+    const int r = u / U, c4 = u % U;
+    *reinterpret_cast<float4*>(dst + (int64_t)r * N + 4 * c4) = *reinterpret_cast<const float4*>(stg + r * LD + 4 * c4);
+  }
+  // the staging tile is generic-proxy data in the region the next stage's TMA writes: every writer
+  // orders its shared-memory stores before those async-proxy writes (CTA-local proxy fence)
+  ptx::fence_proxy_async_smem();
 }
 
 // + bias, then erf-GELU -> bf16 [S][N] (FFN1), or bf16 Q / K head-major and V^T (QKV, the reshape /
@@ -287,8 +302,8 @@ __device__ __forceinline__ void tail_bias(const BertParams& P, const BStage& st,
 
 template <int COLS>
 __device__ __forceinline__ void gemm_tail(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0,
-                                          int split) {
-  if (st.epi == EP_PARTIAL) tail_partial<COLS>(P, st, C, ms, n0, split);
+                                          int split, char* areg) {
+  if (st.epi == EP_PARTIAL) tail_partial<COLS>(P, st, C, ms, n0, split, areg, 3);
   else tail_bias<COLS>(P, st, C, ms, n0);
 }
 
@@ -353,10 +368,10 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
 
   // ---- epilogue (all 8 warps: warp w reads TMEM lanes 32*(w%4).., column half w/4)
   switch (nt) {
-    case 16: gemm_tail<8>(P, st, C, ms, n0, split); break;
-    case 32: gemm_tail<16>(P, st, C, ms, n0, split); break;
-    case 64: gemm_tail<32>(P, st, C, ms, n0, split); break;
-    default: gemm_tail<64>(P, st, C, ms, n0, split); break;
+    case 16: gemm_tail<8>(P, st, C, ms, n0, split, areg); break;
+    case 32: gemm_tail<16>(P, st, C, ms, n0, split, areg); break;
+    case 64: gemm_tail<32>(P, st, C, ms, n0, split, areg); break;
+    default: gemm_tail<64>(P, st, C, ms, n0, split, areg); break;
   }
   if (tid == 0) submark(P, st, 4);
   if (st.fout) flag_signal(st, n0);
@@ -496,13 +511,12 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
     __syncwarp();
     ++ms.wit;
   }
-  if (tid == 0) submark(P, st, 5);
-  // split index = head, N tile = jt (EP_PARTIAL: no bias)
+  // split index = head, N tile = jt (EP_PARTIAL: no bias); staging in the consumed Q/K region
   switch (st.nt) {
-    case 16: tail_partial<8>(P, st, C, ms, jt * st.nt, h); break;
-    case 32: tail_partial<16>(P, st, C, ms, jt * st.nt, h); break;
-    case 64: tail_partial<32>(P, st, C, ms, jt * st.nt, h); break;
-    default: tail_partial<64>(P, st, C, ms, jt * st.nt, h); break;
+    case 16: tail_partial<8>(P, st, C, ms, jt * st.nt, h, areg, 5); break;
+    case 32: tail_partial<16>(P, st, C, ms, jt * st.nt, h, areg, 5); break;
+    case 64: tail_partial<32>(P, st, C, ms, jt * st.nt, h, areg, 5); break;
+    default: tail_partial<64>(P, st, C, ms, jt * st.nt, h, areg, 5); break;
   }
 }
 
@@ -529,13 +543,17 @@ __device__ __forceinline__ float2 block_welford(Ctrl* C, float m, float M2, int 
     C->red[1][w] = M2;
   }
   csync();
-  float mean = C->red[0][0], q = C->red[1][0], na = 128.f;
-  for (int k = 1; k < nwarps; ++k) {
-    const float mb = C->red[0][k], dl = mb - mean;
-    const float nn = na + 128.f;
-    mean += dl * (128.f / nn);
-    q += C->red[1][k] + dl * dl * (na * 128.f / nn);
-    na = nn;
+  // merge warp k (128 values) into warps 0..k-1 (128 k values): mean += dl / (k+1),
+  // M2 += M2_k + dl^2 * 128 k / (k+1)
+  float mean = C->red[0][0], q = C->red[1][0];
+#pragma unroll
+  for (int k = 1; k < 8; ++k) {
+    if (k < nwarps) {
+      const float dl = C->red[0][k] - mean;
+      const float f = 1.f / (float)(k + 1);   // constant-folded
+      mean += dl * f;
+      q += C->red[1][k] + dl * dl * (128.f * (float)k * f);
+    }
   }
   return make_float2(mean, q);
 }
@@ -545,14 +563,12 @@ constexpr int kMaxSplit = 12;   // split-K partials summed by a LayerNorm row
 // pointers, so the later stages (which read the packed copy: a few 2 MB pages instead of ~200
 // scattered allocations) always see the current parameter values
 __device__ void refresh_consts(const BertParams& P) {
-  const int G = gridDim.x * BERT_COMPUTE;
-  int e = 0;
-  for (int i = blockIdx.x * BERT_COMPUTE + threadIdx.x; i < P.copy_total; i += G) {
-    while (e + 1 < P.ncopies && __ldg(&P.copies[e + 1].first) <= i) ++e;
+  for (int e = blockIdx.x; e < P.ncopies; e += gridDim.x) {   // one vector per CTA (n % 4 == 0)
     const BCopy* cp = P.copies + e;
-    const int k = i - __ldg(&cp->first);
-    float* dst = (float*)__ldg(reinterpret_cast<const unsigned long long*>(&cp->dst));
-    dst[k] = __ldg(reinterpret_cast<const float*>(ldgp(&cp->src)) + k);
+    const float4* src = reinterpret_cast<const float4*>(ldgp(&cp->src));
+    float4* dst = (float4*)__ldg(reinterpret_cast<const unsigned long long*>(&cp->dst));
+    const int n4 = __ldg(&cp->n) >> 2;
+    for (int k = threadIdx.x; k < n4; k += BERT_COMPUTE) dst[k] = __ldg(src + k);
   }
 }
 

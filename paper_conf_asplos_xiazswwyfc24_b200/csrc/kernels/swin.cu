@@ -1,0 +1,545 @@
+// Swin-Transformer pattern kernels on sm_100a (B200): the fused subprograms of a Swin block
+// (Table 2), see csrc/swin_types.h for the op list.
+//
+//   sw_gemm_kernel  persistent tcgen05 GEMM: warp 0 streams A / W K-chunks by TMA through a ring,
+//                   warp 1 issues tcgen05.mma (M = 128, N = BN <= 256, K = 16) into one of two TMEM
+//                   accumulators, warps 2-5 run the fused epilogue of the previous tile meanwhile
+//   sw_attn_kernel  window attention, two (window, head) units per M = 128 tile (QK^T, bias + mask,
+//                   softmax in fp32 registers, PV) -- the reductions of Fig. 1(c) kept on chip
+//   sw_row_kernel   LayerNorm of rows gathered through the block's quasi-affine index maps
+//   sw_im2col_kernel, sw_head_kernel   patch embedding gather; final LN + mean pool + classifier
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+#include <algorithm>
+
+#include "../swin_types.h"
+#include "ptx.cuh"
+
+namespace souffle {
+namespace swin {
+
+struct alignas(64) GemmArgs {
+  CUtensorMap ta, tb;
+  SwGemm g;
+};
+struct alignas(64) AttnArgs {
+  CUtensorMap tq, tk, tv;
+  SwAttn a;
+};
+
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+__device__ __forceinline__ uint16_t bf16_bits(float a) {
+  __nv_bfloat16 b = __float2bfloat16_rn(a);
+  return *reinterpret_cast<uint16_t*>(&b);
+}
+__device__ __forceinline__ float bf2f(uint16_t b) { return __uint_as_float(((uint32_t)b) << 16); }
+__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.f + erff(x * 0.70710678118654752f)); }
+__device__ __forceinline__ uint32_t sw128(int row, int kbyte) {
+  return (uint32_t)(row * 128 + ((((kbyte >> 4) ^ (row & 7)) & 7) << 4) + (kbyte & 15));
+}
+
+// K-major operand tile with 64-byte swizzle (rows of 32 bf16): 8-row groups 512 B apart
+__device__ __forceinline__ uint64_t sdesc_sw64(uint32_t saddr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)1 << 16;
+  d |= (uint64_t)(512 >> 4) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)4 << 61;   // SWIZZLE_64B
+  return d;
+}
+
+// ================================================================== GEMM
+// 32 consecutive accumulator columns [n, n + 32) of row r (r < M) through the fused epilogue
+__device__ __forceinline__ void epi_chunk(const SwGemm& g, int r, int n, float* v) {
+  if (g.bias) {
+    const float4* bp = reinterpret_cast<const float4*>(g.bias + n);
+#pragma unroll
+    for (int c = 0; c < 32; c += 4) {
+      const float4 b = __ldg(bp + c / 4);
+      v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
+    }
+  }
+  if (g.epi == SWE_F32) {
+    float4* dst = reinterpret_cast<float4*>(g.out_f + (int64_t)r * g.N + n);
+#pragma unroll
+    for (int c = 0; c < 32; c += 4) dst[c / 4] = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+  } else if (g.epi == SWE_GELU) {
+    uint4* dst = reinterpret_cast<uint4*>(g.out_b + (int64_t)r * g.N + n);
+#pragma unroll
+    for (int c = 0; c < 32; c += 8)
+      dst[c / 8] = make_uint4(pack_bf16(gelu_erf(v[c]), gelu_erf(v[c + 1])), pack_bf16(gelu_erf(v[c + 2]), gelu_erf(v[c + 3])),
+                              pack_bf16(gelu_erf(v[c + 4]), gelu_erf(v[c + 5])), pack_bf16(gelu_erf(v[c + 6]), gelu_erf(v[c + 7])));
+  } else if (g.epi == SWE_RESID) {
+    const int tok = g.rowmap ? __ldg(g.rowmap + r) : r;
+    float4* xp = reinterpret_cast<float4*>(g.out_f + (int64_t)tok * g.N + n);
+    float4 x[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) x[c] = xp[c];
+#pragma unroll
+    for (int c = 0; c < 8; ++c)
+      xp[c] = make_float4(x[c].x + v[4 * c], x[c].y + v[4 * c + 1], x[c].z + v[4 * c + 2], x[c].w + v[4 * c + 3]);
+  } else {   // SWE_QKV: the 32 columns are one head of q, k or v
+    const int which = n / g.C, head = (n % g.C) >> 5;
+    const int win = r / g.L2, i = r % g.L2;
+    const int64_t unit = (int64_t)win * g.heads + head;
+    if (which == 2) {
+      uint16_t* dst = g.vt + unit * (32 * SW_WIN_ROWS) + i;
+#pragma unroll
+      for (int c = 0; c < 32; ++c) dst[c * SW_WIN_ROWS] = bf16_bits(v[c]);
+    } else {
+      const float s = which == 0 ? g.qscale : 1.f;
+      uint4* dst = reinterpret_cast<uint4*>((which == 0 ? g.q : g.k) + (unit * SW_WIN_ROWS + i) * 32);
+#pragma unroll
+      for (int c = 0; c < 32; c += 8)
+        dst[c / 8] = make_uint4(pack_bf16(v[c] * s, v[c + 1] * s), pack_bf16(v[c + 2] * s, v[c + 3] * s),
+                                pack_bf16(v[c + 4] * s, v[c + 5] * s), pack_bf16(v[c + 6] * s, v[c + 7] * s));
+    }
+  }
+}
+
+struct GemmCtrl {
+  uint64_t full[8], empty[8], tfull[2], tempty[2];
+  uint32_t tmem;
+};
+
+__global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __grid_constant__ GemmArgs A) {
+  extern __shared__ __align__(1024) char smem_raw[];
+  char* smem = (char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  GemmCtrl* C = reinterpret_cast<GemmCtrl*>(smem);
+  char* ring = smem + 1024;
+  const SwGemm& g = A.g;
+  const int BN = g.BN, NS = g.stages;
+  const uint32_t A_BYTES = 16384, STAGE = A_BYTES + (uint32_t)BN * 128;
+  const int ntn = g.N / BN, tiles = ntn * ((g.M + 127) / 128), nk = g.K / 64;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) {
+      ptx::mbar_init(&C->full[i], 1);
+      ptx::mbar_init(&C->empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&C->tfull[i], 1);
+      ptx::mbar_init(&C->tempty[i], 128);
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc(&C->tmem, (uint32_t)(2 * BN));
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = C->tmem;
+
+  if (warp == 0) {
+    // ---- TMA producer: A [128 x 64] and W [BN x 64] K-chunks of every tile of this CTA
+    if (lane == 0) {
+      ptx::prefetch_tmap(&A.ta);
+      ptx::prefetch_tmap(&A.tb);
+    }
+    uint32_t it = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
+      const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
+      for (int kc = 0; kc < nk; ++kc, ++it) {
+        const uint32_t slot = it % NS, ph = (it / NS) & 1;
+        ptx::mbar_wait(&C->empty[slot], ph ^ 1);
+        if (ptx::elect_one()) {
+          char* st = ring + slot * STAGE;
+          ptx::mbar_arrive_expect_tx(&C->full[slot], STAGE);
+          ptx::tma_load_2d(st, &A.ta, &C->full[slot], kc * 64, m0);
+          ptx::tma_load_2d(st + A_BYTES, &A.tb, &C->full[slot], kc * 64, n0);
+        }
+        __syncwarp();
+      }
+    }
+  } else if (warp == 1) {
+    // ---- MMA issuer: the whole warp runs the loop (uniform descriptors), one lane issues
+    const uint32_t idesc = ptx::idesc_bf16(128, BN);
+    const uint64_t d0 = ptx::sdesc_sw128(ptx::smem_u32(ring));
+    uint32_t it = 0, lt = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+      const uint32_t buf = lt & 1, use = lt >> 1;
+      ptx::mbar_wait(&C->tempty[buf], (use & 1) ^ 1);
+      ptx::tc_fence_after();
+      const uint32_t d = tmem + buf * BN;
+      for (int kc = 0; kc < nk; ++kc, ++it) {
+        const uint32_t slot = it % NS, ph = (it / NS) & 1;
+        ptx::mbar_wait(&C->full[slot], ph);
+        ptx::tc_fence_after();
+        const uint64_t da = d0 + (uint64_t)((slot * STAGE) >> 4);
+        const uint64_t db = da + (uint64_t)(A_BYTES >> 4);
+        if (ptx::elect_one()) {
+          ptx::mma_bf16_k64(d, da, db, idesc, kc > 0 ? 1u : 0u);
+          ptx::mma_commit(&C->empty[slot]);
+          if (kc == nk - 1) ptx::mma_commit(&C->tfull[buf]);
+        }
+        __syncwarp();
+      }
+    }
+  } else {
+    // ---- epilogue warps 2-5: warp w reads TMEM lanes 32 * (w % 4) .. (its lane quarter)
+    const int q = warp & 3;
+    uint32_t lt = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+      const uint32_t buf = lt & 1, use = lt >> 1;
+      const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
+      ptx::mbar_wait(&C->tfull[buf], use & 1);
+      ptx::tc_fence_after();
+      const int r = m0 + q * 32 + lane;
+      for (int c0 = 0; c0 < BN; c0 += 32) {
+        float v[32];
+        ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
+        if (r < g.M) epi_chunk(g, r, n0 + c0, v);
+      }
+      ptx::tc_fence_before();
+      ptx::mbar_arrive(&C->tempty[buf]);
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) ptx::tmem_dealloc(tmem, (uint32_t)(2 * BN));
+}
+
+// ================================================================== window attention
+struct AttnCtrl {
+  uint64_t ld[2], mma;
+  uint32_t tmem;
+};
+constexpr int kAttnTile = 8192;   // Q pair, K pair, V^T pair: 8 KB each
+
+__global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_constant__ AttnArgs A) {
+  extern __shared__ __align__(1024) char smem_raw[];
+  char* smem = (char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  AttnCtrl* C = reinterpret_cast<AttnCtrl*>(smem);
+  char* Ps = smem + 1024;                      // [128 rows][128 keys] bf16: 2 SW128 atoms of 16 KB
+  char* tiles = Ps + 32768;                    // 2 buffers x (Q, K, V^T)
+  const SwAttn& a = A.a;
+  const int pairs = a.units / 2;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  if (tid == 0) {
+    ptx::mbar_init(&C->ld[0], 1);
+    ptx::mbar_init(&C->ld[1], 1);
+    ptx::mbar_init(&C->mma, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 0) ptx::tmem_alloc(&C->tmem, 256);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = C->tmem;   // S: columns [0, 128); O: [128, 160)
+  auto issue = [&](int p, int b) {
+    char* t = tiles + b * 3 * kAttnTile;
+    ptx::mbar_arrive_expect_tx(&C->ld[b], 3 * kAttnTile);
+    ptx::tma_load_2d(t, &A.tq, &C->ld[b], 0, p * 128);
+    ptx::tma_load_2d(t + kAttnTile, &A.tk, &C->ld[b], 0, p * 128);
+    ptx::tma_load_2d(t + 2 * kAttnTile, &A.tv, &C->ld[b], 0, p * 64);
+  };
+  if (tid == 0 && (int)blockIdx.x < pairs) issue(blockIdx.x, 0);
+  const int r = tid, uh = r >> 6, i = r & 63;   // row of the tile: unit half, token in the window
+  uint32_t it = 0, mph = 0;
+  const float L2E = 1.4426950408889634f;
+  for (int p = blockIdx.x; p < pairs; p += gridDim.x, ++it) {
+    const int b = it & 1;
+    char* t = tiles + b * 3 * kAttnTile;
+    if (tid == 0 && p + (int)gridDim.x < pairs) issue(p + gridDim.x, b ^ 1);   // next pair's tiles
+    ptx::mbar_wait(&C->ld[b], (it >> 1) & 1);
+    // ---- S = Q K^T: M = 128 (two units), N = 128 keys, K = 32 (two K = 16 steps of 32 bytes)
+    if (warp == 0) {
+      ptx::tc_fence_after();
+      const uint64_t dq = sdesc_sw64(ptx::smem_u32(t)), dk = sdesc_sw64(ptx::smem_u32(t + kAttnTile));
+      if (ptx::elect_one()) {
+        ptx::mma_bf16(tmem, dq, dk, ptx::idesc_bf16(128, 128), 0u);
+        ptx::mma_bf16(tmem, dq + 2, dk + 2, ptx::idesc_bf16(128, 128), 1u);
+        ptx::mma_commit(&C->mma);
+      }
+      __syncwarp();
+    }
+    const int unit = 2 * p + uh, win = unit / a.heads, head = unit % a.heads;
+    // bias / mask rows of this thread (issued before the MMA completes)
+    const float* brow = a.bias + ((int64_t)head * a.L2 + i) * a.L2;
+    const float* mrow = a.mask ? a.mask + ((int64_t)(win % a.nW) * a.L2 + i) * a.L2 : nullptr;
+    ptx::mbar_wait(&C->mma, mph);
+    mph ^= 1;
+    ptx::tc_fence_after();
+    float s[64];
+    ptx::tmem_ld64(tmem + ((uint32_t)(warp * 32) << 16) + uh * 64, s);
+    const bool live = i < a.L2;
+    float mx = -INFINITY;
+#pragma unroll
+    for (int j = 0; j < 64; ++j) {
+      if (live && j < a.L2) {
+        float add = __ldg(brow + j);
+        if (mrow) add += __ldg(mrow + j);
+        s[j] = (s[j] + add) * L2E;
+      } else {
+        s[j] = -INFINITY;
+      }
+      mx = fmaxf(mx, s[j]);
+    }
+    float z = 0.f;
+    if (live) {
+#pragma unroll
+      for (int j = 0; j < 64; ++j) {
+        s[j] = ptx::ex2(s[j] - mx);
+        z += s[j];
+      }
+    }
+    const float iz = live ? 1.f / z : 0.f;
+    // P row r: this unit's 64 keys in atom uh, zeros in the other atom (block-diagonal pair)
+#pragma unroll
+    for (int c0 = 0; c0 < 64; c0 += 8) {
+      *reinterpret_cast<uint4*>(Ps + uh * 16384 + sw128(r, c0 * 2)) =
+          live ? make_uint4(pack_bf16(s[c0] * iz, s[c0 + 1] * iz), pack_bf16(s[c0 + 2] * iz, s[c0 + 3] * iz),
+                            pack_bf16(s[c0 + 4] * iz, s[c0 + 5] * iz), pack_bf16(s[c0 + 6] * iz, s[c0 + 7] * iz))
+               : make_uint4(0u, 0u, 0u, 0u);
+      *reinterpret_cast<uint4*>(Ps + (uh ^ 1) * 16384 + sw128(r, c0 * 2)) = make_uint4(0u, 0u, 0u, 0u);
+    }
+    ptx::tc_fence_before();
+    ptx::fence_proxy_async_smem();
+    __syncthreads();
+    // ---- O = P V: M = 128, N = 32, K = 128 keys (atom 0 = unit A's keys with its V^T, atom 1 = B's)
+    if (warp == 0) {
+      ptx::tc_fence_after();
+      const uint64_t dp = ptx::sdesc_sw128(ptx::smem_u32(Ps)), dv = ptx::sdesc_sw128(ptx::smem_u32(t + 2 * kAttnTile));
+      if (ptx::elect_one()) {
+        ptx::mma_bf16_k64(tmem + 128, dp, dv, ptx::idesc_bf16(128, 32), 0u);
+        ptx::mma_bf16_k64(tmem + 128, dp + (16384 >> 4), dv + (4096 >> 4), ptx::idesc_bf16(128, 32), 1u);
+        ptx::mma_commit(&C->mma);
+      }
+      __syncwarp();
+    }
+    ptx::mbar_wait(&C->mma, mph);
+    mph ^= 1;
+    ptx::tc_fence_after();
+    float o[32];
+    ptx::tmem_ld32(tmem + 128 + ((uint32_t)(warp * 32) << 16), o);
+    ptx::tc_fence_before();
+    if (live) {
+      uint4* dst = reinterpret_cast<uint4*>(a.ctx + ((int64_t)win * a.L2 + i) * a.C + head * 32);
+#pragma unroll
+      for (int c = 0; c < 32; c += 8)
+        dst[c / 8] = make_uint4(pack_bf16(o[c], o[c + 1]), pack_bf16(o[c + 2], o[c + 3]), pack_bf16(o[c + 4], o[c + 5]),
+                                pack_bf16(o[c + 6], o[c + 7]));
+    }
+    __syncthreads();   // S / O / P reused by the next pair
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 0) ptx::tmem_dealloc(tmem, 256);
+}
+
+// ================================================================== LayerNorm of gathered rows
+// One warp per output row; lane l holds float4 column groups l, l + 32, ... (NV groups).  The
+// statistics are merged pairwise (Chan) from exactly centred per-lane values: a constant row gives
+// exactly beta, an offset row keeps its noise (no E[x^2] - E[x]^2 cancellation).
+template <int NV>
+__global__ void __launch_bounds__(SW_ROW_THREADS) sw_row_kernel(const SwRow R) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int r = blockIdx.x * (SW_ROW_THREADS / 32) + warp;
+  if (r >= R.rows) return;
+  const int cin = R.cols / R.nsrc;
+  float4 v[NV];
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    const int e = 4 * (lane + 32 * k);
+    const int s = e / cin, o = e - s * cin;
+    const int tok = R.src ? __ldg(R.src + (int64_t)r * R.nsrc + s) : r;
+    v[k] = __ldg(reinterpret_cast<const float4*>(R.x + (int64_t)tok * cin + o));
+  }
+  float m = 0.f;
+#pragma unroll
+  for (int k = 0; k < NV; ++k) m += (v[k].x + v[k].y) + (v[k].z + v[k].w);
+  m *= 1.f / (float)(4 * NV);
+  float M2 = 0.f;
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    const float a = v[k].x - m, b = v[k].y - m, c = v[k].z - m, d = v[k].w - m;
+    M2 += (a * a + b * b) + (c * c + d * d);
+  }
+  float n = (float)(4 * NV);
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const float mb = __shfl_xor_sync(0xffffffffu, m, o), Mb = __shfl_xor_sync(0xffffffffu, M2, o);
+    const float dl = mb - m;
+    M2 = (M2 + Mb) + dl * dl * (0.5f * n);
+    m = (m + mb) * 0.5f;
+    n *= 2.f;
+  }
+  const float rs = rsqrtf(M2 / (float)R.cols + R.eps);
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    const int e = 4 * (lane + 32 * k);
+    const float4 gm = __ldg(reinterpret_cast<const float4*>(R.gamma + e));
+    const float4 bt = __ldg(reinterpret_cast<const float4*>(R.beta + e));
+    const float4 y = make_float4((v[k].x - m) * rs * gm.x + bt.x, (v[k].y - m) * rs * gm.y + bt.y,
+                                 (v[k].z - m) * rs * gm.z + bt.z, (v[k].w - m) * rs * gm.w + bt.w);
+    if (R.out_b)
+      *reinterpret_cast<uint2*>(R.out_b + (int64_t)r * R.cols + e) = make_uint2(pack_bf16(y.x, y.y), pack_bf16(y.z, y.w));
+    if (R.out_f) *reinterpret_cast<float4*>(R.out_f + (int64_t)r * R.cols + e) = y;
+  }
+}
+
+// ================================================================== patch embedding gather
+__global__ void sw_im2col_kernel(const SwIm2col P) {
+  const int64_t T = (int64_t)P.B * P.R * P.R;
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx < (int64_t)P.C * 64) {   // padded weight copy [C][64]
+    const int row = (int)(idx / 64), col = (int)(idx % 64);
+    P.wpad[idx] = col < 48 ? P.w[row * 48 + col] : (uint16_t)0;
+  }
+  if (idx >= T * 64) return;
+  const int col = (int)(idx % 64);
+  const int64_t tok = idx / 64;
+  float v = 0.f;
+  if (col < 3 * P.p * P.p) {
+    const int b = (int)(tok / (P.R * P.R)), ty = (int)(tok / P.R % P.R), tx = (int)(tok % P.R);
+    const int c = col / (P.p * P.p), kh = col / P.p % P.p, kw = col % P.p;
+    v = __ldg(P.image + (((int64_t)b * 3 + c) * P.img + ty * P.p + kh) * P.img + tx * P.p + kw);
+  }
+  P.out[idx] = bf16_bits(v);
+}
+
+// ================================================================== final LN + mean pool + head
+__global__ void __launch_bounds__(256) sw_head_kernel(const SwHead H) {
+  extern __shared__ float hsm[];          // [8][C] per-warp pooled sums, then [C] bf16-rounded mean
+  const int b = blockIdx.x, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int C = H.C, NV = C / 128;
+  for (int c = threadIdx.x; c < 8 * C; c += 256) hsm[c] = 0.f;
+  __syncthreads();
+  for (int t = warp; t < H.L; t += 8) {
+    const float* xr = H.x + ((int64_t)b * H.L + t) * C;
+    float4 v[8];
+    float m = 0.f;
+    for (int k = 0; k < NV; ++k) {
+      v[k] = __ldg(reinterpret_cast<const float4*>(xr) + lane + 32 * k);
+      m += (v[k].x + v[k].y) + (v[k].z + v[k].w);
+    }
+    m *= 1.f / (float)(4 * NV);
+    float M2 = 0.f, n = (float)(4 * NV);
+    for (int k = 0; k < NV; ++k) {
+      const float a = v[k].x - m, bb = v[k].y - m, c = v[k].z - m, d = v[k].w - m;
+      M2 += (a * a + bb * bb) + (c * c + d * d);
+    }
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float mb = __shfl_xor_sync(0xffffffffu, m, o), Mb = __shfl_xor_sync(0xffffffffu, M2, o);
+      const float dl = mb - m;
+      M2 = (M2 + Mb) + dl * dl * (0.5f * n);
+      m = (m + mb) * 0.5f;
+      n *= 2.f;
+    }
+    const float rs = rsqrtf(M2 / (float)C + H.eps);
+    for (int k = 0; k < NV; ++k) {
+      const int e = 4 * (lane + 32 * k);
+      const float4 gm = __ldg(reinterpret_cast<const float4*>(H.gamma + e));
+      const float4 bt = __ldg(reinterpret_cast<const float4*>(H.beta + e));
+      float* p = hsm + warp * C + e;
+      p[0] += (v[k].x - m) * rs * gm.x + bt.x;
+      p[1] += (v[k].y - m) * rs * gm.y + bt.y;
+      p[2] += (v[k].z - m) * rs * gm.z + bt.z;
+      p[3] += (v[k].w - m) * rs * gm.w + bt.w;
+    }
+  }
+  __syncthreads();
+  float* pooled = hsm + 8 * C;   // bf16-rounded mean (the classifier matmul has bf16 operands)
+  for (int c = threadIdx.x; c < C; c += 256) {
+    float s = 0.f;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) s += hsm[w * C + c];
+    pooled[c] = bf2f(bf16_bits(s / (float)H.L));
+  }
+  __syncthreads();
+  for (int n = warp; n < H.classes; n += 8) {
+    const uint16_t* wr = H.W + (int64_t)n * C;
+    float acc = 0.f;
+    for (int c = lane * 8; c < C; c += 256) {
+      const uint4 w8 = __ldg(reinterpret_cast<const uint4*>(wr + c));
+      const uint32_t ws[4] = {w8.x, w8.y, w8.z, w8.w};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        acc += pooled[c + 2 * j] * __uint_as_float(ws[j] << 16);
+        acc += pooled[c + 2 * j + 1] * __uint_as_float(ws[j] & 0xffff0000u);
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) H.out[(int64_t)b * H.classes + n] = acc + __ldg(H.bias + n);
+  }
+}
+
+}  // namespace swin
+
+// ------------------------------------------------------------------ host-side launchers
+// dynamic shared-memory opt-in, once per kernel (the largest configuration any launch uses)
+static cudaError_t set_smem(const void* f, int bytes) {
+  static const void* done[8] = {};
+  for (const void* d : done)
+    if (d == f) return cudaSuccess;
+  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess)
+    for (auto& d : done)
+      if (!d) { d = f; break; }
+  return e;
+}
+
+int sw_gemm_smem(int BN, int stages) { return 2048 + stages * (16384 + BN * 128); }
+int sw_attn_smem() { return 2048 + 32768 + 2 * 3 * swin::kAttnTile; }
+
+cudaError_t sw_launch_gemm(const void* ta, const void* tb, const SwGemm& g, int grid, cudaStream_t s) {
+  swin::GemmArgs a;
+  memcpy(&a.ta, ta, sizeof(CUtensorMap));
+  memcpy(&a.tb, tb, sizeof(CUtensorMap));
+  a.g = g;
+  const int sm = sw_gemm_smem(g.BN, g.stages);
+  cudaError_t e = set_smem((const void*)swin::sw_gemm_kernel, 227 * 1024);
+  if (e != cudaSuccess) return e;
+  swin::sw_gemm_kernel<<<grid, SW_GEMM_THREADS, sm, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t sw_launch_attn(const void* tq, const void* tk, const void* tv, const SwAttn& at, int grid, cudaStream_t s) {
+  swin::AttnArgs a;
+  memcpy(&a.tq, tq, sizeof(CUtensorMap));
+  memcpy(&a.tk, tk, sizeof(CUtensorMap));
+  memcpy(&a.tv, tv, sizeof(CUtensorMap));
+  a.a = at;
+  const int sm = sw_attn_smem();
+  cudaError_t e = set_smem((const void*)swin::sw_attn_kernel, sm);
+  if (e != cudaSuccess) return e;
+  swin::sw_attn_kernel<<<grid, SW_ATTN_THREADS, sm, s>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t sw_launch_row(const SwRow& r, cudaStream_t s) {
+  const int grid = (r.rows + 7) / 8;
+  switch (r.cols / 128) {
+    case 1: swin::sw_row_kernel<1><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
+    case 2: swin::sw_row_kernel<2><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
+    case 4: swin::sw_row_kernel<4><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
+    case 8: swin::sw_row_kernel<8><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
+    case 16: swin::sw_row_kernel<16><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t sw_launch_im2col(const SwIm2col& p, cudaStream_t s) {
+  const int64_t n = std::max<int64_t>((int64_t)p.B * p.R * p.R * 64, (int64_t)p.C * 64);
+  swin::sw_im2col_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t sw_launch_head(const SwHead& h, cudaStream_t s) {
+  const int sm = (9 * h.C) * 4;
+  cudaError_t e = set_smem((const void*)swin::sw_head_kernel, 9 * 1024 * 4);
+  if (e != cudaSuccess) return e;
+  swin::sw_head_kernel<<<h.B, 256, sm, s>>>(h);
+  return cudaGetLastError();
+}
+
+}  // namespace souffle

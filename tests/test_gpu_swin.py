@@ -55,23 +55,49 @@ def test_swin_tiny_bf16_tensor_cores():
     assert np.max(np.abs(again - ref)) <= 2e-2
 
 
-def _swin_b_child():
-    got, again, ref, plan = _run(S.SWIN_B, bf16=True)
-    print("RESULT", got.shape[0], got.shape[1], float(np.max(np.abs(got - ref))), float(np.max(np.abs(again - ref))))
+# the Swin pattern kernels (kernels/swin.cu): head dim 32, window 7, C % 128 == 0.  56 x 56 images
+# give a 14 x 14 stage (2 x 2 windows, shifted blocks with the mask), a patch merge and a 7 x 7
+# stage whose window covers the map (no shift) -- every kernel and index map of the pattern
+SWIN_PAT = dict(S.SWIN_TINY, embed=128, heads=(4, 8), gemm_dtype="bf16")
 
 
-def test_swin_b_batch1_full_size():
-    """Full Swin-B at batch 1 against the bf16-operand oracle, in a fresh process (isolated from the
-    kernels the other tests ran; this is how a stall fixed this round was first contained)."""
+@pytest.mark.parametrize("batch", [1, 3])
+def test_swin_pattern_small(batch, record_err):
+    got, again, ref, plan = _run(dict(SWIN_PAT, batch=batch), bf16=True)
+    assert "pattern swin: batch" in plan.describe()
+    record_err(float(np.max(np.abs(got - ref))), 2e-2, batch=batch, rms=float(np.sqrt(np.mean(ref ** 2))))
+    assert np.array_equal(got, again)          # no atomics on the data path: bit-reproducible
+
+
+def test_swin_pattern_generic_agree():
+    """The pattern kernels and the generic fused executor compute the same TE program."""
+    cfg = dict(SWIN_PAT, batch=2)
+    got, _, ref, plan = _run(cfg, bf16=True)
+    gen, _, _, gplan = _run(cfg, flags=L.FLAG_NO_PATTERN, bf16=True)
+    assert "pattern swin: batch" in plan.describe() and "pattern swin: not used" in gplan.describe()
+    assert np.max(np.abs(got - gen)) <= 2e-2
+
+
+def _swin_b_child(batch):
+    got, again, ref, plan = _run(dict(S.SWIN_B, batch=batch), bf16=True)
+    print("RESULT", got.shape[0], got.shape[1], float(np.max(np.abs(got - ref))), float(np.max(np.abs(again - ref))),
+          float(np.sqrt(np.mean(ref ** 2))), "pattern swin: batch" in plan.describe())
+
+
+@pytest.mark.parametrize("batch", [1, 8])
+def test_swin_b_full_size(batch, record_err):
+    """Full Swin-B (BASELINE.json configs[4]) at batch 1 and 8 through the pattern kernels against the
+    bf16-operand oracle, in a fresh process (isolated from the kernels the other tests ran)."""
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    code = "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_swin as t; t._swin_b_child()" % (
-        root, os.path.join(root, "tests"))
-    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, cwd=root)
+    code = "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_swin as t; t._swin_b_child(%d)" % (
+        root, os.path.join(root, "tests"), batch)
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=900, cwd=root)
     line = [ln for ln in r.stdout.splitlines() if ln.startswith("RESULT")]
     assert line, r.stderr[-2000:]
-    _, b, n, e1, e2 = line[0].split()
-    assert (int(b), int(n)) == (1, 1000)
-    assert float(e1) <= 2e-2 and float(e2) <= 2e-2, (e1, e2)
+    _, b, n, e1, e2, rms, pat = line[0].split()
+    assert (int(b), int(n)) == (batch, 1000) and pat == "True"
+    assert float(e2) <= 2e-2
+    record_err(float(e1), 2e-2, batch=batch, rms=float(rms))
