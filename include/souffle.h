@@ -220,7 +220,9 @@ souffle_status souffle_plan_read_profile_raw(souffle_plan p, void* workspace, ui
  * [2*heads][S][64]), "vt" (bf16 V^T [heads][64][S]), "h" (bf16 GELU output [S][F]), "part_o" /
  * "part_2" (fp32 split-K partials [nsplit][S][H]).  Used with SOUFFLE_BERT_STAGES=b,e (run only
  * stages [b, e)) by the stage-isolation tests.  Errors: E_INVALID_ARG (unknown name, NULL
- * pointers), E_UNSUPPORTED (the plan does not use the BERT pattern kernel). */
+ * pointers), E_UNSUPPORTED (the plan does not use the BERT pattern kernel).  A Swin pattern plan
+ * has one region, "trace": one uint64 %globaltimer stamp per launch (CTA 0, after its dependency
+ * wait) when the workspace was initialised with SOUFFLE_SWIN_TRACE set. */
 souffle_status souffle_plan_debug_region(souffle_plan p, const char* name, int64_t* offset, int64_t* bytes);
 
 #ifdef __cplusplus

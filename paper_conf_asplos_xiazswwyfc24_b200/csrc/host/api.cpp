@@ -442,6 +442,11 @@ souffle_status souffle_plan_debug_region(souffle_plan p, const char* name, int64
     Plan& P = PL(p);
     if (!name || !offset || !bytes) throw Error(SOUFFLE_E_INVALID_ARG, "null argument");
     const BertPlan& b = P.bert;
+    if (P.swin.on && std::string(name) == "trace") {   // Swin debug trace: one u64 stamp per launch
+      *offset = P.swin.o_trace;
+      *bytes = 8 * (int64_t)P.swin.launches;
+      return;
+    }
     if (!b.on) throw Error(SOUFFLE_E_UNSUPPORTED, "the plan does not use the BERT pattern kernel");
     const int64_t S = b.S, H = b.H, F = b.F;
     const std::string n(name);

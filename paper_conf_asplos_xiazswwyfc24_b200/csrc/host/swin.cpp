@@ -33,6 +33,8 @@ cudaError_t sw_launch_attn(const void* tq, const void* tk, const void* tv, const
 cudaError_t sw_launch_row(const SwRow& r, cudaStream_t s);
 cudaError_t sw_launch_im2col(const SwIm2col& p, cudaStream_t s);
 cudaError_t sw_launch_head(const SwHead& h, cudaStream_t s);
+cudaError_t sw_launch_bias(const SwBias& b, int max_table, cudaStream_t s);
+cudaError_t sw_launch_pool(const SwHead& h, cudaStream_t s);
 
 namespace {
 
@@ -279,7 +281,7 @@ void swin_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   if (!c.ok || c.i != N.size() || ef != eps) return no("TE program is not a Swin Transformer");
   if (g.outputs.size() != 1 || g.outputs[0] != y) return no("the only output must be the logits");
   if (sp.blocks.empty() || (int)sp.merges.size() + 1 != (int)sp.depths.size()) return no("stage structure");
-  if (3 * p * p > 64 || C0 % 128 || C > 1024 || 4 * (C / 2) > 2048) return no("patch size / widths");
+  if (p != 4 || C0 % 128 || C > 1024 || 4 * (C / 2) > 2048) return no("patch size 4 / widths");
   sp.B = (int)B; sp.img = (int)img; sp.patch = (int)p; sp.C0 = (int)C0; sp.window = (int)w;
   sp.classes = (int)classes; sp.eps = eps; sp.X = 0; sp.Y = y;
   sp.num_sms = dev.num_sms > 0 ? dev.num_sms : 148;
@@ -301,6 +303,25 @@ void swin_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   sp.o_k = take(qk * 2);
   sp.o_vt = take(qk * 2);
   sp.o_wpad = take(C0 * 64 * 2);
+  sp.o_pool = take(B * 1024 * 4);
+  sp.o_trace = take(8 * 1024);
+  // split-K partials / counters (a split GEMM has at most num_sms units of 128 x 256 fp32)
+  sp.o_part = take((int64_t)sp.num_sms * 128 * 256 * 4);
+  sp.o_cnt = take((int64_t)2 * sp.num_sms * 4 + 256);
+  // per-block score-bias tables [nW or 1][heads][SW_TAB] (rebuilt from the bound bias / mask by the
+  // first launch of every run) and their descriptor list
+  {
+    int64_t tabs = 0, Rr = R;
+    size_t gb = 0;
+    for (size_t s2 = 0; s2 < sp.depths.size(); ++s2, Rr /= 2)
+      for (int j = 0; j < sp.depths[s2]; ++j, ++gb) {
+        const int64_t nWe = sp.blocks[gb].mask >= 0 ? (Rr / w) * (Rr / w) : 1;
+        tabs += nWe * sp.heads[s2] * SW_TAB;
+      }
+    sp.o_tab = take(tabs * 4);
+    sp.tab_floats = tabs;
+    sp.o_tabent = take((int64_t)sp.blocks.size() * (int64_t)sizeof(SwBiasEnt));
+  }
   // index maps: per stage the unshifted and shifted window maps, then the merge maps
   sp.maps.clear();
   {
@@ -385,16 +406,64 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
   const int32_t* maps = (const int32_t*)(base + sp.o_maps);
   ops.clear();
   tm.clear();
+  float* tabs = (float*)(base + sp.o_tab);
+  SwBiasEnt* tabent = (SwBiasEnt*)(base + sp.o_tabent);
+  std::vector<float*> block_tab;
+  std::vector<int> block_nw;
+  {
+    SwinOp op;
+    op.kind = SW_BIAS;
+    int64_t off = 0, Rr = R1;
+    size_t gb2 = 0;
+    sp.tabent.clear();
+    for (size_t s2 = 0; s2 < sp.depths.size(); ++s2, Rr /= 2)
+      for (int j = 0; j < sp.depths[s2]; ++j, ++gb2) {
+        const SwinBlockIds& bk = sp.blocks[gb2];
+        SwBiasEnt e{};
+        e.bias = fptr(bk.bias);
+        e.mask = bk.mask >= 0 ? fptr(bk.mask) : nullptr;
+        e.dst = tabs + off;
+        e.heads = sp.heads[s2];
+        e.nW = bk.mask >= 0 ? (int)((Rr / w) * (Rr / w)) : 1;
+        e.first = (int32_t)off;
+        sp.tabent.push_back(e);
+        block_tab.push_back(tabs + off);
+        block_nw.push_back(e.nW);
+        off += (int64_t)e.nW * e.heads * SW_TAB;
+      }
+    int64_t mx = 0;
+    for (auto& e : sp.tabent) mx = std::max<int64_t>(mx, (int64_t)e.nW * e.heads * SW_TAB);
+    op.grid = (int)std::min<int64_t>(mx, 1 << 30);   // largest table (elements): sizes the launch
+    op.bias.ent = tabent;
+    op.bias.n = (int)sp.tabent.size();
+    op.bias.total = (int32_t)off;
+    op.bias.L2 = L2;
+    ops.push_back(op);
+    tm.push_back(Launcher{});
+  }
   auto gemm = [&](void* A, int64_t M, int64_t K, void* W, int64_t N, int epi) -> SwinOp& {
     SwinOp op;
     op.kind = SW_GEMM;
     SwGemm& g = op.gemm;
     std::memset(&g, 0, sizeof(g));
     g.M = (int)M; g.N = (int)N; g.K = (int)K; g.epi = epi;
-    g.BN = N % 256 == 0 ? 256 : N % 128 == 0 ? 128 : 64;
+    // tile policy: the widest N tile (smem operand bandwidth per MMA) that still fills the SMs;
+    // with too few output tiles (small M, e.g. batch 1) the K loop is split across CTAs
+    const int64_t mt = (M + 127) / 128, nk = K / 64;
+    g.BN = 64;
+    for (int bn : {256, 128}) {
+      if (N % bn == 0 && mt * (N / bn) >= nsm) { g.BN = bn; break; }
+    }
+    if (g.BN == 64 && N % 64) g.BN = N % 128 == 0 ? 128 : 256;
     g.stages = g.BN == 256 ? 4 : g.BN == 128 ? 6 : 8;
-    const int tiles = (int)(N / g.BN) * (int)((M + 127) / 128);
-    op.grid = std::min(tiles, nsm);
+    const int tiles = (int)(N / g.BN * mt);
+    g.splits = 1;
+    if (tiles * 2 <= nsm)
+      for (int sp2 = 16; sp2 >= 2; sp2 >>= 1)
+        if (nk % sp2 == 0 && tiles * sp2 <= nsm) { g.splits = sp2; break; }
+    g.part = (float*)(base + sp.o_part);
+    g.cnt = (unsigned*)(base + sp.o_cnt);
+    op.grid = g.splits > 1 ? tiles * g.splits : std::min(tiles, nsm);
     Launcher L;
     if (!make_map(&L.maps[0], A, M, K, 128, 64, 128) || !make_map(&L.maps[1], W, N, K, g.BN, 64, 128)) op.grid = -1;
     ops.push_back(op);
@@ -444,8 +513,8 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
         SwinOp op;
         op.kind = SW_ATTN;
         SwAttn& a = op.attn;
-        a.units = (int)units; a.heads = (int)nh; a.nW = (int)nW; a.L2 = L2;
-        a.bias = fptr(bk.bias); a.mask = bk.mask >= 0 ? fptr(bk.mask) : nullptr; a.ctx = ctx; a.C = (int)C;
+        a.units = (int)units; a.heads = (int)nh; a.nW = block_nw[gb]; a.L2 = L2;
+        a.tab = block_tab[gb]; a.ctx = ctx; a.C = (int)C;
         op.grid = (int)std::min<int64_t>(units / 2, 2 * nsm);
         Launcher L;
         if (!make_map(&L.maps[0], qb, units * 64, 32, 128, 32, 64) || !make_map(&L.maps[1], kb, units * 64, 32, 128, 32, 64) ||
@@ -477,15 +546,24 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
       R /= 2;
     }
   }
-  {
+  for (int k : {SW_POOL, SW_HEAD}) {
     SwinOp op;
-    op.kind = SW_HEAD;
+    op.kind = k;
     SwHead& hd = op.head;
     hd.B = B; hd.L = (int)(R * R); hd.C = (int)C; hd.classes = sp.classes; hd.x = x[cur];
     hd.gamma = fptr(sp.gn); hd.beta = fptr(sp.ben); hd.eps = (float)sp.eps;
     hd.W = (const uint16_t*)bound(sp.Wh); hd.bias = fptr(sp.bh); hd.out = (float*)bound(sp.Y);
+    hd.pooled = (float*)(base + sp.o_pool);
     ops.push_back(op);
     tm.push_back(Launcher{});
+  }
+  // debug trace (SOUFFLE_SWIN_TRACE=1): every launch stamps %globaltimer into the workspace
+  unsigned long long* tr = std::getenv("SOUFFLE_SWIN_TRACE") ? (unsigned long long*)(base + sp.o_trace) : nullptr;
+  for (size_t i = 0; i < ops.size(); ++i) {
+    SwinOp& op = ops[i];
+    const int k = (int)i;
+    op.gemm.trace = op.attn.trace = op.row.trace = op.im2col.trace = op.head.trace = op.bias.trace = tr;
+    op.gemm.op = op.attn.op = op.row.op = op.im2col.op = op.head.op = op.bias.op = k;
   }
   for (auto& op : ops)
     if (op.grid < 0) return fail(SOUFFLE_E_CUDA, "cuTensorMapEncodeTiled failed (pointer alignment?)");
@@ -501,6 +579,8 @@ static cudaError_t launch_ops(const std::vector<SwinOp>& ops, const std::vector<
       case SW_ROW: e = sw_launch_row(op.row, s); break;
       case SW_GEMM: e = sw_launch_gemm(&tm[i].maps[0], &tm[i].maps[1], op.gemm, op.grid, s); break;
       case SW_ATTN: e = sw_launch_attn(&tm[i].maps[0], &tm[i].maps[1], &tm[i].maps[2], op.attn, op.grid, s); break;
+      case SW_BIAS: e = sw_launch_bias(op.bias, op.grid, s); break;
+      case SW_POOL: e = sw_launch_pool(op.head, s); break;
       default: e = sw_launch_head(op.head, s); break;
     }
   }
@@ -518,6 +598,9 @@ souffle_status swin_init(Plan& p, void* ws, void* stream) {
   cudaError_t e = cudaMemsetAsync(base, 0, (size_t)sp.total, s);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(base + sp.o_maps, sp.maps.data(), sp.maps.size() * 4, cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(base + sp.o_tabent, sp.tabent.data(), sp.tabent.size() * sizeof(SwBiasEnt),
+                        cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("swin workspace init: ") + cudaGetErrorString(e));
   // capture the launch sequence once (kernel parameters hold the tensor maps and pointers)
@@ -556,7 +639,7 @@ souffle_status swin_run(Plan& p, void* ws, void* stream) {
 }
 
 int swin_launch_count(const SwinPlan& sp) {
-  int n = 3 + 1;   // im2col, embed GEMM, embed LN, head
+  int n = 4 + 2;   // bias tables, im2col, embed GEMM, embed LN; pool, head
   for (size_t s = 0; s < sp.depths.size(); ++s) n += 7 * sp.depths[s] + (s + 1 < sp.depths.size() ? 2 : 0);
   return n;
 }

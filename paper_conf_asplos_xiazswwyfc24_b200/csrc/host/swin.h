@@ -31,6 +31,7 @@ struct SwinOp {
   SwRow row{};
   SwIm2col im2col{};
   SwHead head{};
+  SwBias bias{};
   int grid = 0;
   // tensor map requests: (buffer id, rows, cols, box rows, box cols, swizzle bytes); buffer ids are
   // workspace offsets (>= 0) or -(node + 1) for a bound tensor
@@ -50,7 +51,8 @@ struct SwinPlan {
   std::vector<SwinMergeIds> merges;
   // workspace layout (byte offsets)
   int64_t o_x0 = 0, o_x1 = 0, o_a = 0, o_ctx = 0, o_h = 0, o_q = 0, o_k = 0, o_vt = 0, o_pe = 0, o_wpad = 0;
-  int64_t o_maps = 0, total = 0;
+  int64_t o_maps = 0, o_tab = 0, o_tabent = 0, tab_floats = 0, o_pool = 0, o_trace = 0, o_part = 0, o_cnt = 0, total = 0;
+  std::vector<SwBiasEnt> tabent;   // score-bias table descriptors (pointers resolved at init)
   std::vector<int32_t> maps;    // host copy of the int32 index maps (uploaded at init)
   std::vector<SwinOp> ops;      // launch sequence (pointers resolved at init)
   int launches = 0;

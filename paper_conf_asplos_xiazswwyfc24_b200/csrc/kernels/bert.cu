@@ -99,12 +99,20 @@ __device__ __forceinline__ void spin_guard(uint32_t& n, unsigned long long& t0) 
 // ------------------------------------------------------------------ grid barrier (split phase)
 __device__ __forceinline__ void grid_arrive(const BertParams& P, int k, bool tma_consumed) {
   // generic-proxy writes of this stage -> TMA reads of later stages (split-K partials are read by
-  // plain loads of the LayerNorm rows: no proxy fence for those stages)
-  if (tma_consumed) ptx::fence_proxy_async();
+  // plain loads of the LayerNorm rows: no proxy fence for those stages).  The data is global: the
+  // proxy fence is restricted to the global state space (timing study bit 1 << 20: full fence)
+  if (tma_consumed) {
+    if (P.dbg_skip & (1 << 20)) ptx::fence_proxy_async();
+    else ptx::fence_proxy_async_global();
+  }
   csync();
   if (threadIdx.x == 0) {
-    __threadfence();
-    atomicAdd(&P.ctrl[k], 1u);
+    if (P.dbg_skip & (1 << 21)) {
+      __threadfence();
+      atomicAdd(&P.ctrl[k], 1u);
+    } else {
+      ptx::red_release_add(&P.ctrl[k], 1u);   // release: orders the CTA's writes (bar.sync above) first
+    }
   }
 }
 __device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target_arrivals, bool tma_reads) {
@@ -113,7 +121,7 @@ __device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target
     uint32_t n = 0;
     unsigned long long t0 = 0;
     while (ptx::ld_acquire(&P.ctrl[k]) < target) spin_guard(n, t0);
-    if (tma_reads) ptx::fence_proxy_async();   // the stage reads other CTAs' data through TMA
+    if (tma_reads) ptx::fence_proxy_async_global();   // the stage reads other CTAs' data through TMA
   }
   csync();
 }

@@ -44,6 +44,20 @@ __device__ __forceinline__ uint32_t sw128(int row, int kbyte) {
   return (uint32_t)(row * 128 + ((((kbyte >> 4) ^ (row & 7)) & 7) << 4) + (kbyte & 15));
 }
 
+// programmatic dependent launch: let the next kernel of the stream start its prologue now, and wait
+// for the previous kernel's completion (and memory) before touching global memory
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// debug trace: CTA 0 stamps %globaltimer when launch `op` passes its dependency wait
+__device__ __forceinline__ void trace_stamp(unsigned long long* tr, int op) {
+  if (tr && blockIdx.x == 0 && blockIdx.y == 0 && threadIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    tr[op] = t;
+  }
+}
+__device__ __forceinline__ void epi_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+
 // K-major operand tile with 64-byte swizzle (rows of 32 bf16): 8-row groups 512 B apart
 __device__ __forceinline__ uint64_t sdesc_sw64(uint32_t saddr) {
   uint64_t d = 0;
@@ -115,10 +129,12 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
   GemmCtrl* C = reinterpret_cast<GemmCtrl*>(smem);
   char* ring = smem + 1024;
   const SwGemm& g = A.g;
-  const int BN = g.BN, NS = g.stages;
+  const int BN = g.BN, NS = g.stages, SP = g.splits;
   const uint32_t A_BYTES = 16384, STAGE = A_BYTES + (uint32_t)BN * 128;
-  const int ntn = g.N / BN, tiles = ntn * ((g.M + 127) / 128), nk = g.K / 64;
+  const int ntn = g.N / BN, tiles = ntn * ((g.M + 127) / 128), nk = g.K / 64 / SP;   // chunks per unit
+  const int units = tiles * SP;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  pdl_trigger();
   if (threadIdx.x == 0) {
     for (int i = 0; i < NS; ++i) {
       ptx::mbar_init(&C->full[i], 1);
@@ -126,24 +142,27 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
     }
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&C->tfull[i], 1);
-      ptx::mbar_init(&C->tempty[i], 128);
+      ptx::mbar_init(&C->tempty[i], 256);
     }
     ptx::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    ptx::prefetch_tmap(&A.ta);
+    ptx::prefetch_tmap(&A.tb);
   }
   if (warp == 1) ptx::tmem_alloc(&C->tmem, (uint32_t)(2 * BN));
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = C->tmem;
+  pdl_wait();   // the A operand / residual stream is written by the previous kernel
+  trace_stamp(g.trace, g.op);
 
   if (warp == 0) {
-    // ---- TMA producer: A [128 x 64] and W [BN x 64] K-chunks of every tile of this CTA
-    if (lane == 0) {
-      ptx::prefetch_tmap(&A.ta);
-      ptx::prefetch_tmap(&A.tb);
-    }
+    // ---- TMA producer: A [128 x 64] and W [BN x 64] K-chunks of every unit of this CTA
     uint32_t it = 0;
-    for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
+    for (int u = blockIdx.x; u < units; u += gridDim.x) {
+      const int t = u / SP, kc0 = (u % SP) * nk;
       const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
       for (int kc = 0; kc < nk; ++kc, ++it) {
         const uint32_t slot = it % NS, ph = (it / NS) & 1;
@@ -151,8 +170,8 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
         if (ptx::elect_one()) {
           char* st = ring + slot * STAGE;
           ptx::mbar_arrive_expect_tx(&C->full[slot], STAGE);
-          ptx::tma_load_2d(st, &A.ta, &C->full[slot], kc * 64, m0);
-          ptx::tma_load_2d(st + A_BYTES, &A.tb, &C->full[slot], kc * 64, n0);
+          ptx::tma_load_2d(st, &A.ta, &C->full[slot], (kc0 + kc) * 64, m0);
+          ptx::tma_load_2d(st + A_BYTES, &A.tb, &C->full[slot], (kc0 + kc) * 64, n0);
         }
         __syncwarp();
       }
@@ -162,7 +181,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
     const uint32_t idesc = ptx::idesc_bf16(128, BN);
     const uint64_t d0 = ptx::sdesc_sw128(ptx::smem_u32(ring));
     uint32_t it = 0, lt = 0;
-    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+    for (int u = blockIdx.x; u < units; u += gridDim.x, ++lt) {
       const uint32_t buf = lt & 1, use = lt >> 1;
       ptx::mbar_wait(&C->tempty[buf], (use & 1) ^ 1);
       ptx::tc_fence_after();
@@ -182,22 +201,65 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       }
     }
   } else {
-    // ---- epilogue warps 2-5: warp w reads TMEM lanes 32 * (w % 4) .. (its lane quarter)
-    const int q = warp & 3;
+    // ---- epilogue warps 2-9: warp w reads TMEM lanes 32 * (w % 4) .. (its lane quarter); the two
+    // warps of a quarter take alternate 32-column chunks
+    const int q = warp & 3, eh = (warp - 2) >> 2, et = threadIdx.x - 64;
     uint32_t lt = 0;
-    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++lt) {
+    for (int u = blockIdx.x; u < units; u += gridDim.x, ++lt) {
       const uint32_t buf = lt & 1, use = lt >> 1;
+      const int t = u / SP, split = u % SP;
       const int m0 = (t / ntn) * 128, n0 = (t % ntn) * BN;
       ptx::mbar_wait(&C->tfull[buf], use & 1);
       ptx::tc_fence_after();
-      const int r = m0 + q * 32 + lane;
-      for (int c0 = 0; c0 < BN; c0 += 32) {
+      const int rt = q * 32 + lane, r = m0 + rt;
+      for (int c0 = 32 * eh; c0 < BN; c0 += 64) {
         float v[32];
         ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
-        if (r < g.M) epi_chunk(g, r, n0 + c0, v);
+        if (SP == 1) {
+          if (r < g.M) epi_chunk(g, r, n0 + c0, v);
+        } else {   // fp32 partial of this split
+          float4* dst = reinterpret_cast<float4*>(g.part + ((int64_t)u * 128 + rt) * BN + c0);
+#pragma unroll
+          for (int c = 0; c < 32; c += 4) dst[c / 4] = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+        }
       }
       ptx::tc_fence_before();
       ptx::mbar_arrive(&C->tempty[buf]);
+      if (SP > 1) {
+        // meet the other splits of this tile (all units are co-resident: grid == units <= #SMs)
+        __threadfence();
+        epi_sync();
+        if (et == 0) {
+          atomicAdd(&g.cnt[t], 1u);
+          while (ptx::ld_acquire(&g.cnt[t]) < (unsigned)SP) {
+          }
+        }
+        epi_sync();
+        // reduce rows [split * 128 / SP, ...) of the tile, splits summed in order
+        const int rows = 128 / SP, cpr = BN / 32;
+        for (int item = et; item < rows * cpr; item += 256) {
+          const int rr = split * rows + item / cpr, c0 = (item % cpr) * 32;
+          float v[32];
+#pragma unroll
+          for (int c = 0; c < 32; ++c) v[c] = 0.f;
+          for (int k = 0; k < SP; ++k) {
+            const float4* src = reinterpret_cast<const float4*>(g.part + ((int64_t)(t * SP + k) * 128 + rr) * BN + c0);
+#pragma unroll
+            for (int c = 0; c < 32; c += 4) {
+              const float4 x = __ldcg(src + c / 4);
+              v[c] += x.x; v[c + 1] += x.y; v[c + 2] += x.z; v[c + 3] += x.w;
+            }
+          }
+          if (m0 + rr < g.M) epi_chunk(g, m0 + rr, n0 + c0, v);
+        }
+        epi_sync();
+        if (et == 0) {   // the last split to finish resets the tile's counters for the next run
+          if (atomicAdd(&g.cnt[tiles + t], 1u) == (unsigned)SP - 1) {
+            g.cnt[t] = 0u;
+            g.cnt[tiles + t] = 0u;
+          }
+        }
+      }
     }
   }
   ptx::tc_fence_before();
@@ -207,10 +269,11 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
 
 // ================================================================== window attention
 struct AttnCtrl {
-  uint64_t ld[2], mma;
+  uint64_t ld[2], mma, tb;
   uint32_t tmem;
 };
 constexpr int kAttnTile = 8192;   // Q pair, K pair, V^T pair: 8 KB each
+constexpr int kTabBytes = 2 * SW_TAB * 4;   // the pair's two score-bias tiles
 
 __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_constant__ AttnArgs A) {
   extern __shared__ __align__(1024) char smem_raw[];
@@ -218,13 +281,16 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
   AttnCtrl* C = reinterpret_cast<AttnCtrl*>(smem);
   char* Ps = smem + 1024;                      // [128 rows][128 keys] bf16: 2 SW128 atoms of 16 KB
   char* tiles = Ps + 32768;                    // 2 buffers x (Q, K, V^T)
+  float* tab = reinterpret_cast<float*>(tiles + 2 * 3 * kAttnTile);   // the pair's score-bias tiles
   const SwAttn& a = A.a;
   const int pairs = a.units / 2;
   const int tid = threadIdx.x, warp = tid >> 5;
+  pdl_trigger();
   if (tid == 0) {
     ptx::mbar_init(&C->ld[0], 1);
     ptx::mbar_init(&C->ld[1], 1);
     ptx::mbar_init(&C->mma, 1);
+    ptx::mbar_init(&C->tb, 1);
     ptx::fence_mbar_init();
   }
   if (warp == 0) ptx::tmem_alloc(&C->tmem, 256);
@@ -232,6 +298,8 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = C->tmem;   // S: columns [0, 128); O: [128, 160)
+  pdl_wait();
+  trace_stamp(a.trace, a.op);
   auto issue = [&](int p, int b) {
     char* t = tiles + b * 3 * kAttnTile;
     ptx::mbar_arrive_expect_tx(&C->ld[b], 3 * kAttnTile);
@@ -239,7 +307,18 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
     ptx::tma_load_2d(t + kAttnTile, &A.tk, &C->ld[b], 0, p * 128);
     ptx::tma_load_2d(t + 2 * kAttnTile, &A.tv, &C->ld[b], 0, p * 64);
   };
-  if (tid == 0 && (int)blockIdx.x < pairs) issue(blockIdx.x, 0);
+  // the pair's two (window, head) tiles of the score-bias table: units 2p, 2p+1 are heads h, h+1 of
+  // one window, contiguous in tab[window % nW][heads]
+  auto issue_tab = [&](int p) {
+    const int unit = 2 * p, win = unit / a.heads, head = unit % a.heads;
+    const float* src = a.tab + ((int64_t)(win % a.nW) * a.heads + head) * SW_TAB;
+    ptx::mbar_arrive_expect_tx(&C->tb, kTabBytes);
+    ptx::bulk_g2s(tab, src, kTabBytes, &C->tb);
+  };
+  if (tid == 0 && (int)blockIdx.x < pairs) {
+    issue(blockIdx.x, 0);
+    issue_tab(blockIdx.x);
+  }
   const int r = tid, uh = r >> 6, i = r & 63;   // row of the tile: unit half, token in the window
   uint32_t it = 0, mph = 0;
   const float L2E = 1.4426950408889634f;
@@ -260,9 +339,8 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
       __syncwarp();
     }
     const int unit = 2 * p + uh, win = unit / a.heads, head = unit % a.heads;
-    // bias / mask rows of this thread (issued before the MMA completes)
-    const float* brow = a.bias + ((int64_t)head * a.L2 + i) * a.L2;
-    const float* mrow = a.mask ? a.mask + ((int64_t)(win % a.nW) * a.L2 + i) * a.L2 : nullptr;
+    const float* trow = tab + uh * SW_TAB + i * a.L2;   // this row's additive terms (smem)
+    ptx::mbar_wait(&C->tb, it & 1);
     ptx::mbar_wait(&C->mma, mph);
     mph ^= 1;
     ptx::tc_fence_after();
@@ -273,9 +351,7 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
 #pragma unroll
     for (int j = 0; j < 64; ++j) {
       if (live && j < a.L2) {
-        float add = __ldg(brow + j);
-        if (mrow) add += __ldg(mrow + j);
-        s[j] = (s[j] + add) * L2E;
+        s[j] = (s[j] + trow[j]) * L2E;
       } else {
         s[j] = -INFINITY;
       }
@@ -302,6 +378,8 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
     ptx::tc_fence_before();
     ptx::fence_proxy_async_smem();
     __syncthreads();
+    // the table is consumed: fetch the next pair's (it lands during PV and the stores)
+    if (tid == 0 && p + (int)gridDim.x < pairs) issue_tab(p + gridDim.x);
     // ---- O = P V: M = 128, N = 32, K = 128 keys (atom 0 = unit A's keys with its V^T, atom 1 = B's)
     if (warp == 0) {
       ptx::tc_fence_after();
@@ -340,6 +418,9 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
 template <int NV>
 __global__ void __launch_bounds__(SW_ROW_THREADS) sw_row_kernel(const SwRow R) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  pdl_trigger();
+  pdl_wait();
+  trace_stamp(R.trace, R.op);
   const int r = blockIdx.x * (SW_ROW_THREADS / 32) + warp;
   if (r >= R.rows) return;
   const int cin = R.cols / R.nsrc;
@@ -384,29 +465,58 @@ __global__ void __launch_bounds__(SW_ROW_THREADS) sw_row_kernel(const SwRow R) {
   }
 }
 
+// ================================================================== score-bias tables
+__global__ void sw_bias_kernel(const SwBias B) {
+  pdl_trigger();
+  pdl_wait();
+  trace_stamp(B.trace, B.op);
+  const SwBiasEnt& E = B.ent[blockIdx.y];
+  const int L2 = B.L2;
+  const int64_t n = (int64_t)E.nW * E.heads * SW_TAB;
+  for (int64_t o = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; o < n; o += (int64_t)gridDim.x * blockDim.x) {
+    const int t = (int)(o % SW_TAB);
+    const int64_t u = o / SW_TAB;           // (w, h) unit of the table
+    const int h = (int)(u % E.heads), w = (int)(u / E.heads);
+    float v = 0.f;
+    if (t < L2 * L2) {
+      v = __ldg(E.bias + (int64_t)h * L2 * L2 + t);
+      if (E.mask) v += __ldg(E.mask + (int64_t)w * L2 * L2 + t);
+    }
+    E.dst[o] = v;
+  }
+}
+
 // ================================================================== patch embedding gather
+// thread per (token, 4-column group): groups 0..11 = (c, kh) rows of the 4 x 4 patch (one float4 of
+// the image row), 12..15 = zero padding of K to 64
 __global__ void sw_im2col_kernel(const SwIm2col P) {
+  pdl_trigger();
+  pdl_wait();
+  trace_stamp(P.trace, P.op);
   const int64_t T = (int64_t)P.B * P.R * P.R;
   const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (idx < (int64_t)P.C * 64) {   // padded weight copy [C][64]
     const int row = (int)(idx / 64), col = (int)(idx % 64);
     P.wpad[idx] = col < 48 ? P.w[row * 48 + col] : (uint16_t)0;
   }
-  if (idx >= T * 64) return;
-  const int col = (int)(idx % 64);
-  const int64_t tok = idx / 64;
-  float v = 0.f;
-  if (col < 3 * P.p * P.p) {
+  if (idx >= T * 16) return;
+  const int g = (int)(idx % 16);
+  const int64_t tok = idx / 16;
+  float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (g < 12) {
     const int b = (int)(tok / (P.R * P.R)), ty = (int)(tok / P.R % P.R), tx = (int)(tok % P.R);
-    const int c = col / (P.p * P.p), kh = col / P.p % P.p, kw = col % P.p;
-    v = __ldg(P.image + (((int64_t)b * 3 + c) * P.img + ty * P.p + kh) * P.img + tx * P.p + kw);
+    const int c = g >> 2, kh = g & 3;
+    v = __ldg(reinterpret_cast<const float4*>(P.image + (((int64_t)b * 3 + c) * P.img + ty * 4 + kh) * P.img + tx * 4));
   }
-  P.out[idx] = bf16_bits(v);
+  reinterpret_cast<uint2*>(P.out)[idx] = make_uint2(pack_bf16(v.x, v.y), pack_bf16(v.z, v.w));
 }
 
 // ================================================================== final LN + mean pool + head
-__global__ void __launch_bounds__(256) sw_head_kernel(const SwHead H) {
-  extern __shared__ float hsm[];          // [8][C] per-warp pooled sums, then [C] bf16-rounded mean
+__global__ void __launch_bounds__(256) sw_pool_kernel(const SwHead H) {
+  extern __shared__ float hsm[];          // [8][C] per-warp pooled sums
+  pdl_trigger();
+  pdl_wait();
+  trace_stamp(H.trace, H.op);
   const int b = blockIdx.x, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int C = H.C, NV = C / 128;
   for (int c = threadIdx.x; c < 8 * C; c += 256) hsm[c] = 0.f;
@@ -446,35 +556,82 @@ __global__ void __launch_bounds__(256) sw_head_kernel(const SwHead H) {
     }
   }
   __syncthreads();
-  float* pooled = hsm + 8 * C;   // bf16-rounded mean (the classifier matmul has bf16 operands)
   for (int c = threadIdx.x; c < C; c += 256) {
     float s = 0.f;
 #pragma unroll
     for (int w = 0; w < 8; ++w) s += hsm[w * C + c];
-    pooled[c] = bf2f(bf16_bits(s / (float)H.L));
+    H.pooled[(int64_t)b * C + c] = bf2f(bf16_bits(s / (float)H.L));   // bf16 matmul operand
   }
-  __syncthreads();
-  for (int n = warp; n < H.classes; n += 8) {
-    const uint16_t* wr = H.W + (int64_t)n * C;
-    float acc = 0.f;
-    for (int c = lane * 8; c < C; c += 256) {
-      const uint4 w8 = __ldg(reinterpret_cast<const uint4*>(wr + c));
-      const uint32_t ws[4] = {w8.x, w8.y, w8.z, w8.w};
+}
+
+// a warp per class: the class's weight row stays in registers, dotted with every image's pooled row
+__global__ void __launch_bounds__(256) sw_head_kernel(const SwHead H) {
+  pdl_trigger();
+  pdl_wait();
+  trace_stamp(H.trace, H.op);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n = blockIdx.x * 8 + warp;
+  if (n >= H.classes) return;
+  const int C = H.C;
+  float w[32];   // C <= 1024: 32 weights per lane, columns lane * 8 + 256 * j + e
+  const uint16_t* wr = H.W + (int64_t)n * C;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    uint4 w8 = make_uint4(0u, 0u, 0u, 0u);
+    if (lane * 8 + 256 * j < C) w8 = __ldg(reinterpret_cast<const uint4*>(wr + lane * 8 + 256 * j));
+    const uint32_t ws[4] = {w8.x, w8.y, w8.z, w8.w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      w[8 * j + 2 * e] = __uint_as_float(ws[e] << 16);
+      w[8 * j + 2 * e + 1] = __uint_as_float(ws[e] & 0xffff0000u);
+    }
+  }
+  const float bias = __ldg(H.bias + n);
+  for (int b0 = 0; b0 < H.B; b0 += 4) {   // 4 images at a time: independent loads in flight
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+    for (int bb = 0; bb < 4; ++bb) {
+      if (b0 + bb >= H.B) break;
+      const float* pr = H.pooled + (int64_t)(b0 + bb) * C;
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        acc += pooled[c + 2 * j] * __uint_as_float(ws[j] << 16);
-        acc += pooled[c + 2 * j + 1] * __uint_as_float(ws[j] & 0xffff0000u);
+        if (lane * 8 + 256 * j < C) {
+          const float4 p0 = __ldcg(reinterpret_cast<const float4*>(pr + lane * 8 + 256 * j));
+          const float4 p1 = __ldcg(reinterpret_cast<const float4*>(pr + lane * 8 + 256 * j + 4));
+          acc[bb] += p0.x * w[8 * j] + p0.y * w[8 * j + 1] + p0.z * w[8 * j + 2] + p0.w * w[8 * j + 3] +
+                     p1.x * w[8 * j + 4] + p1.y * w[8 * j + 5] + p1.z * w[8 * j + 6] + p1.w * w[8 * j + 7];
+        }
       }
     }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (lane == 0) H.out[(int64_t)b * H.classes + n] = acc + __ldg(H.bias + n);
+    for (int bb = 0; bb < 4; ++bb) {
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) acc[bb] += __shfl_xor_sync(0xffffffffu, acc[bb], o);
+      if (lane == 0 && b0 + bb < H.B) H.out[(int64_t)(b0 + bb) * H.classes + n] = acc[bb] + bias;
+    }
   }
 }
 
 }  // namespace swin
 
 // ------------------------------------------------------------------ host-side launchers
+// every launch allows programmatic dependent launch: the next kernel's CTAs start (prologue: barrier
+// init, TMEM alloc, tensor-map prefetch) while this one drains, and wait in griddepcontrol.wait
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args&&... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
+}
+
 // dynamic shared-memory opt-in, once per kernel (the largest configuration any launch uses)
 static cudaError_t set_smem(const void* f, int bytes) {
   static const void* done[8] = {};
@@ -488,18 +645,16 @@ static cudaError_t set_smem(const void* f, int bytes) {
 }
 
 int sw_gemm_smem(int BN, int stages) { return 2048 + stages * (16384 + BN * 128); }
-int sw_attn_smem() { return 2048 + 32768 + 2 * 3 * swin::kAttnTile; }
+int sw_attn_smem() { return 2048 + 32768 + 2 * 3 * swin::kAttnTile + swin::kTabBytes; }
 
 cudaError_t sw_launch_gemm(const void* ta, const void* tb, const SwGemm& g, int grid, cudaStream_t s) {
   swin::GemmArgs a;
   memcpy(&a.ta, ta, sizeof(CUtensorMap));
   memcpy(&a.tb, tb, sizeof(CUtensorMap));
   a.g = g;
-  const int sm = sw_gemm_smem(g.BN, g.stages);
   cudaError_t e = set_smem((const void*)swin::sw_gemm_kernel, 227 * 1024);
   if (e != cudaSuccess) return e;
-  swin::sw_gemm_kernel<<<grid, SW_GEMM_THREADS, sm, s>>>(a);
-  return cudaGetLastError();
+  return launch_pdl(swin::sw_gemm_kernel, dim3(grid), dim3(SW_GEMM_THREADS), (size_t)sw_gemm_smem(g.BN, g.stages), s, a);
 }
 
 cudaError_t sw_launch_attn(const void* tq, const void* tk, const void* tv, const SwAttn& at, int grid, cudaStream_t s) {
@@ -511,35 +666,38 @@ cudaError_t sw_launch_attn(const void* tq, const void* tk, const void* tv, const
   const int sm = sw_attn_smem();
   cudaError_t e = set_smem((const void*)swin::sw_attn_kernel, sm);
   if (e != cudaSuccess) return e;
-  swin::sw_attn_kernel<<<grid, SW_ATTN_THREADS, sm, s>>>(a);
-  return cudaGetLastError();
+  return launch_pdl(swin::sw_attn_kernel, dim3(grid), dim3(SW_ATTN_THREADS), (size_t)sm, s, a);
 }
 
 cudaError_t sw_launch_row(const SwRow& r, cudaStream_t s) {
-  const int grid = (r.rows + 7) / 8;
+  const dim3 grid((r.rows + 7) / 8), blk(SW_ROW_THREADS);
   switch (r.cols / 128) {
-    case 1: swin::sw_row_kernel<1><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
-    case 2: swin::sw_row_kernel<2><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
-    case 4: swin::sw_row_kernel<4><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
-    case 8: swin::sw_row_kernel<8><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
-    case 16: swin::sw_row_kernel<16><<<grid, SW_ROW_THREADS, 0, s>>>(r); break;
+    case 1: return launch_pdl(swin::sw_row_kernel<1>, grid, blk, 0, s, r);
+    case 2: return launch_pdl(swin::sw_row_kernel<2>, grid, blk, 0, s, r);
+    case 4: return launch_pdl(swin::sw_row_kernel<4>, grid, blk, 0, s, r);
+    case 8: return launch_pdl(swin::sw_row_kernel<8>, grid, blk, 0, s, r);
+    case 16: return launch_pdl(swin::sw_row_kernel<16>, grid, blk, 0, s, r);
     default: return cudaErrorInvalidValue;
   }
-  return cudaGetLastError();
+}
+
+cudaError_t sw_launch_bias(const SwBias& b, int max_table, cudaStream_t s) {
+  return launch_pdl(swin::sw_bias_kernel, dim3((unsigned)std::min(64, (max_table + 1023) / 1024), b.n), dim3(256), 0, s, b);
 }
 
 cudaError_t sw_launch_im2col(const SwIm2col& p, cudaStream_t s) {
-  const int64_t n = std::max<int64_t>((int64_t)p.B * p.R * p.R * 64, (int64_t)p.C * 64);
-  swin::sw_im2col_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(p);
-  return cudaGetLastError();
+  const int64_t n = std::max<int64_t>((int64_t)p.B * p.R * p.R * 16, (int64_t)p.C * 64);
+  return launch_pdl(swin::sw_im2col_kernel, dim3((unsigned)((n + 255) / 256)), dim3(256), 0, s, p);
+}
+
+cudaError_t sw_launch_pool(const SwHead& h, cudaStream_t s) {
+  cudaError_t e = set_smem((const void*)swin::sw_pool_kernel, 8 * 1024 * 4);
+  if (e != cudaSuccess) return e;
+  return launch_pdl(swin::sw_pool_kernel, dim3(h.B), dim3(256), (size_t)(8 * h.C * 4), s, h);
 }
 
 cudaError_t sw_launch_head(const SwHead& h, cudaStream_t s) {
-  const int sm = (9 * h.C) * 4;
-  cudaError_t e = set_smem((const void*)swin::sw_head_kernel, 9 * 1024 * 4);
-  if (e != cudaSuccess) return e;
-  swin::sw_head_kernel<<<h.B, 256, sm, s>>>(h);
-  return cudaGetLastError();
+  return launch_pdl(swin::sw_head_kernel, dim3((h.classes + 7) / 8), dim3(256), 0, s, h);
 }
 
 }  // namespace souffle

@@ -19,14 +19,16 @@
 
 namespace souffle {
 
-enum SwOpKind : int32_t { SW_IM2COL = 0, SW_ROW = 1, SW_GEMM = 2, SW_ATTN = 3, SW_HEAD = 4 };
+enum SwOpKind : int32_t { SW_IM2COL = 0, SW_ROW = 1, SW_GEMM = 2, SW_ATTN = 3, SW_HEAD = 4, SW_BIAS = 5, SW_POOL = 6 };
 enum SwEpi : int32_t { SWE_F32 = 0, SWE_GELU = 1, SWE_RESID = 2, SWE_QKV = 3 };
 
 enum {
-  SW_GEMM_THREADS = 192,      // warp 0 TMA producer, warp 1 MMA issuer, warps 2-5 epilogue
+  SW_GEMM_THREADS = 320,      // warp 0 TMA producer, warp 1 MMA issuer, warps 2-9 epilogue (2 per
+                              // TMEM lane quarter, alternating 32-column chunks)
   SW_ATTN_THREADS = 128,      // one thread per row of the M = 128 tile (two 64-row units)
   SW_ROW_THREADS = 256,       // 8 warps, one token row per warp
   SW_WIN_ROWS = 64,           // a (window, head) unit: 49 tokens padded to 64 rows
+  SW_TAB = 2404,              // floats per (window, head) score-bias tile: 49 x 49 + 3 (16-byte multiple)
 };
 
 // one GEMM launch: C[M, N] = A[M, K] W[N, K]^T (bf16 operands, fp32 accumulate) + epilogue
@@ -43,15 +45,41 @@ struct SwGemm {
   uint16_t *q, *k, *vt;
   int32_t C, heads, L2;       // L2 = window tokens (49)
   float qscale;
+  // split-K (small M, e.g. batch 1: too few output tiles to occupy the SMs): unit = tile * splits +
+  // split covers K chunks [split * nk / splits, ...); the fp32 partials go to part[unit][128][BN],
+  // the `splits` CTAs of a tile meet on cnt[tile] and each reduces 128 / splits rows (fixed split
+  // order: deterministic) through the fused epilogue; cnt[tiles + tile] counts the finished ones
+  int32_t splits;             // 1 = no split
+  float* part;
+  unsigned* cnt;
+  unsigned long long* trace;  // debug: %globaltimer at the start of launch `op` (CTA 0), or null
+  int32_t op;
 };
 
-// window attention over `units` (window, head) pairs, two per CTA iteration
+// window attention over `units` (window, head) pairs, two per CTA iteration.  The additive score
+// terms come from a per-block table tab[nW][heads][SW_TAB] = relative-position bias (+ shifted-window
+// mask) built by sw_bias_kernel at the start of every run (nW = 1 for unshifted blocks), so a pair's
+// two tiles are one contiguous bulk copy into shared memory
 struct SwAttn {
-  int32_t units, heads, nW, L2; // nW: windows per image (mask index = window % nW)
-  const float* bias;            // [heads][L2][L2] relative-position bias
-  const float* mask;            // [nW][L2][L2] shifted-window mask, or null
+  int32_t units, heads, nW, L2; // nW: windows per image in the table (window index = window % nW)
+  const float* tab;
   uint16_t* ctx;                // bf16 [windows * L2][heads * 32] (window order)
   int32_t C;
+  unsigned long long* trace;
+  int32_t op;
+};
+
+// one block's score-bias table: dst[w][h][i * L2 + j] = bias[h][i][j] + (mask ? mask[w][i][j] : 0)
+struct SwBiasEnt {
+  const float* bias;
+  const float* mask;
+  float* dst;
+  int32_t heads, nW, first, pad;   // first: element offset of this table in the concatenation
+};
+struct SwBias {
+  const SwBiasEnt* ent;
+  int32_t n, total, L2, op;
+  unsigned long long* trace;
 };
 
 // LayerNorm of gathered rows: out[r] = LN(concat_s x[src[r * nsrc + s]]) * gamma + beta
@@ -64,6 +92,8 @@ struct SwRow {
   float eps;
   uint16_t* out_b;              // bf16 [rows][cols] (GEMM A operand), or null
   float* out_f;                 // fp32 [rows][cols], or null
+  unsigned long long* trace;
+  int32_t op;
 };
 
 // patch-embedding im2col: image [B][3][H][W] fp32 -> bf16 [B * R * R][64] (48 used, cols =
@@ -74,9 +104,13 @@ struct SwIm2col {
   uint16_t* out;
   const uint16_t* w;            // bound Wpe [C][48] (bf16)
   uint16_t* wpad;               // [C][64]
+  unsigned long long* trace;
+  int32_t op;
 };
 
-// final LayerNorm + mean over the L tokens of each image + classifier (bf16 operands, fp32 acc)
+// final LayerNorm + mean over the L tokens of each image (sw_pool_kernel, one CTA per image; the
+// mean is rounded to bf16: it is a matmul operand), then the classifier (sw_head_kernel, a warp per
+// class over all images; bf16 operands, fp32 accumulate)
 struct SwHead {
   int32_t B, L, C, classes;
   const float* x;               // fp32 [B * L][C]
@@ -86,6 +120,9 @@ struct SwHead {
   const uint16_t* W;            // bf16 [classes][C]
   const float* bias;            // [classes]
   float* out;                   // fp32 [B][classes]
+  float* pooled;                // fp32 [B][C] workspace (bf16-representable values)
+  unsigned long long* trace;
+  int32_t op;
 };
 
 }  // namespace souffle

@@ -235,7 +235,7 @@ def test_pattern_kernels_follow_the_partition():
 def test_swin_pattern_matches_and_skips_generic_lowering():
     import time
     import synth.swin as S
-    for cfg, launches in ((S.SWIN_B, 178), (dict(S.SWIN_TINY, embed=128, heads=(4, 8), gemm_dtype="bf16"), 34)):
+    for cfg, launches in ((S.SWIN_B, 180), (dict(S.SWIN_TINY, embed=128, heads=(4, 8), gemm_dtype="bf16"), 36)):
         g, names, x, y = M.swin(cfg)
         t0 = time.perf_counter()
         plan = g.partition(L.device_b200())
