@@ -406,6 +406,22 @@ def main():
                                      "activations)", "latency_us": lat, "wavefront_steps": steps_wf,
                          "us_per_wavefront_step": lat / steps_wf, "weight_bytes": lw,
                          "hbm_roofline_us": lw / (hbm * 1e3), "kernel": lplan.describe().splitlines()[1][:160]}
+        # the dependency-chain bound: wavefront steps x the measured one-way
+        # exchange latency between two SMs (tools/bench_exchange.cu, profiles/r02_exchange.json), and
+        # the kernel's pipe utilisation from ncu (profiles/r02_ncu_lstm_pipes.json; Table 6)
+        pe = os.path.join(ROOT, "profiles", "r02_exchange.json")
+        if os.path.exists(pe):
+            ex = json.load(open(pe))
+            cb = steps_wf * ex["t_exchange_min_ns"] / 1e3
+            extra["lstm"].update({"t_exchange_min_ns": ex["t_exchange_min_ns"], "chain_bound_us": cb,
+                                  "chain_bound_frac": cb / lat,
+                                  "chain_bound_source": "profiles/r02_exchange.json (tools/bench_exchange.cu)"})
+        pp = os.path.join(ROOT, "profiles", "r02_ncu_lstm_pipes.json")
+        if os.path.exists(pp):
+            extra["lstm"]["ncu_pipes"] = json.load(open(pp))
+        sys.path.insert(0, os.path.join(ROOT, "tools"))
+        from graph_timing import graph_us
+        extra["lstm"]["graph_replay_us_per_inference"] = graph_us(lsess.run, reps=20, sess=lsess)
         del lsess, lplan
         progress("MMoE")
         mplan, msess = build_mmoe(local)
@@ -432,7 +448,12 @@ def main():
                          "latency_us": statistics.median(tm) * 1e3, "launches": mplan.exec_info()["launches"],
                          "stages": mplan.exec_info()["stages"],
                          "back_to_back_us_per_inference": a.elapsed_time(b) * 1e3 / 100,
-                         "empty_kernel_same_bracket_us": statistics.median(td)}
+                         "empty_kernel_same_bracket_us": statistics.median(td),
+                         # device time: a CUDA graph of 100 inferences replayed (no CPU submission per
+                         # launch); an empty kernel replayed the same way is the per-launch floor
+                         "graph_replay_us_per_inference": graph_us(msess.run, sess=msess),
+                         "empty_kernel_graph_replay_us": graph_us(lambda: dummy.add_(1)),
+                         "paper_a100_us": 14.0}
         del msess, mplan
         # Swin-B runs in a child process (fresh CUDA context) with a time limit: a launch that trips a
         # kernel watchdog must not take the whole bench line with it

@@ -34,7 +34,8 @@ enum {
   BA_SLOT_BYTES = 16384,
   B_CTRL_BYTES = 2048,         // control block + two staged stage descriptors
   B_AREGION = BA_SLOTS * BA_SLOT_BYTES,   // also holds the attention operands Q, K, V^T, P (80 KB)
-  B_SMEM = B_CTRL_BYTES + BW_SLOTS * BW_SLOT_BYTES + B_AREGION + 1024   // + alignment slack
+  B_RECV_BYTES = 16384,        // cluster-pair split-K: the partner's fp32 half tile (128 x <= 32 cols)
+  B_SMEM = B_CTRL_BYTES + BW_SLOTS * BW_SLOT_BYTES + B_AREGION + B_RECV_BYTES + 1024   // + alignment slack
 };
 
 struct alignas(16) BStage {
@@ -61,6 +62,8 @@ struct alignas(16) BStage {
   unsigned int* fout;
   // ---- ROW: mode 0 convert (out_b = bf16(in)); mode 1 LayerNorm(sum_s part[s] + bias + res)
   int32_t row_mode, cols, r_nsplit, arrive;
+  int32_t cpair, pad0, pad1, pad2;   // GEMM nsplit == 2 over a CTA pair (cluster): partial sums
+                                     // exchanged through distributed shared memory (DSMEM)
   const float* r_in;            // mode 0: fp32 [S][cols]; mode 1: partials [r_nsplit][S][cols]
   const float* r_bias;
   const float* r_res;
@@ -90,6 +93,7 @@ struct BertParams {
   const BCopy* copies;          // constant vectors refreshed in stage 0 (all CTAs take part)
   int32_t ncopies, copy_total;  // entries, total floats
   int32_t s_begin, s_end;       // stages executed: [0, nstages) except in stage-isolation tests
+  int32_t pairs;                // launched as CTA-pair clusters (cluster-pair split-K stages)
 };
 
 }  // namespace souffle

@@ -24,7 +24,7 @@ namespace souffle {
 
 extern thread_local std::string g_err;
 souffle_status fail(souffle_status c, const std::string& m);
-cudaError_t bert_launch(const BertParams& prm, int grid, cudaStream_t s);
+cudaError_t bert_launch(const BertParams& prm, int grid, bool pairs, cudaStream_t s);
 cudaError_t bert_max_active(int* blocks);
 
 namespace {
@@ -263,6 +263,22 @@ void bert_match(const Graph& g, const Analysis& an, const souffle_device_desc& d
     if (bp.H % nt == 0 && (bp.H / nt) * bp.heads <= sms) { bp.out = BertGemmCfg{nt, bp.heads, 1, bp.H / nt}; break; }
   if (bp.heads > 12) return no("more than 12 heads (split-K partials summed per LayerNorm row)");
   bp.ffn1 = full_cfg(bp.F, bp.H, sms, 128, "SOUFFLE_BERT_FFN1");
+  // cluster-pair split-K for the full-K GEMMs (QKV, FFN1): a CTA pair splits K in halves and sums
+  // through DSMEM, halving the activation bytes every CTA streams (SOUFFLE_BERT_PAIRS=0 disables)
+  {
+    const char* e = std::getenv("SOUFFLE_BERT_PAIRS");
+    const int kc = bp.H / 64;
+    bp.pairs = (!e || std::atoi(e) != 0) && sms % 2 == 0 && kc % 2 == 0;
+    if (bp.pairs) {
+      const BertGemmCfg q{32, 2, kc / 2, 3 * bp.H / 32}, f{64, 2, kc / 2, bp.F / 64};
+      if (q.tiles_n * 2 <= sms && f.tiles_n * 2 <= sms) {
+        bp.qkv = q;
+        bp.ffn1 = f;
+      } else {
+        bp.pairs = false;
+      }
+    }
+  }
   bp.ffn2 = split_cfg(bp.H, bp.F, sms, "SOUFFLE_BERT_FFN2");
   for (const BertGemmCfg* q : {&bp.qkv, &bp.out, &bp.ffn1, &bp.ffn2})
     if (q->nt == 0 || q->tiles_n * q->nsplit > sms) return no("no tile configuration fits one wave of CTAs");
@@ -301,8 +317,10 @@ std::string bert_describe(const BertPlan& bp) {
     return os.str();
   }
   auto g = [&](const char* nm, const BertGemmCfg& c) {
+    const bool pair = bp.pairs && (&c == &bp.qkv || &c == &bp.ffn1);
     os << "    " << nm << ": n_tile " << c.nt << " x split-K " << c.nsplit << " (" << c.kchunks * 64
-       << " K per task) = " << c.tiles_n * c.nsplit << " tasks\n";
+       << " K per task) = " << c.tiles_n * c.nsplit << " tasks" << (pair ? " (cluster pairs, DSMEM reduction)" : "")
+       << "\n";
   };
   os << "pattern bert: " << bp.layers.size() << " encoder layer(s), S=" << bp.S << " H=" << bp.H << " heads="
      << bp.heads << " F=" << bp.F << " -> 1 persistent launch (kernels/bert.cu), " << bp.nstages << " stages, "
@@ -447,6 +465,7 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
     const int t = kActMaps + 6 * l;
     const float* xin = l == 0 ? X : xf;
     BStage a = gemm(l, bp.qkv, 3 * H, H, t + 0, H, MAP_XB, EP_QKV);
+    a.cpair = bp.pairs ? 1 : 0;
     a.bias = cptr(L.bq);   // bq, bk, bv are packed contiguously: the [Q | K | V] bias
     a.out_b = qk; a.out_vt = vt;
     st.push_back(a);
@@ -465,6 +484,7 @@ souffle_status bert_init(Plan& p, void* ws, void* stream) {
     st.push_back(at);
     st.push_back(ln(l, part_o, bp.out.nsplit, cptr(L.bo), xin, cptr(L.g1), cptr(L.be1), l1f, l1b));
     BStage f1 = gemm(l, bp.ffn1, F, H, t + 4, F, MAP_L1B, EP_GELU);
+    f1.cpair = bp.pairs ? 1 : 0;
     f1.bias = cptr(L.c1); f1.out_b = hb;
     if (p2p_ffn) { f1.fout = fl_ffn; f1.fdiv = bp.ffn2.kchunks * 64; f1.fmod = (int)F; }
     st.push_back(f1);
@@ -548,6 +568,7 @@ souffle_status bert_run(Plan& p, void* ws, void* stream) {
   if (const char* dbg = std::getenv("SOUFFLE_BERT_DBG_SKIP")) prm.dbg_skip = std::atoi(dbg);   // timing studies
   prm.s_begin = 0;
   prm.s_end = bp.nstages;
+  prm.pairs = bp.pairs ? 1 : 0;
   // stage-isolation tests (tests/test_gpu_bert_stages.py): run only stages [b, e) on a workspace the
   // test pre-filled (the integer bit-exact checks of single GEMM stages)
   if (const char* se = std::getenv("SOUFFLE_BERT_STAGES")) {
@@ -557,7 +578,7 @@ souffle_status bert_run(Plan& p, void* ws, void* stream) {
       prm.s_end = en;
     }
   }
-  cudaError_t e = bert_launch(prm, grid, (cudaStream_t)stream);
+  cudaError_t e = bert_launch(prm, grid, bp.pairs, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("bert launch: ") + cudaGetErrorString(e));
   return SOUFFLE_OK;
 }

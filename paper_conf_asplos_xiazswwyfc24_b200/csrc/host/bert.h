@@ -33,6 +33,7 @@ struct BertPlan {
   std::vector<BertLayerIds> layers;
   BertGemmCfg qkv, out, ffn1, ffn2;
   int num_sms = 0;
+  bool pairs = false;             // QKV / FFN1 as cluster-pair split-K (kernels/bert.cu pair_tail)
   int nstages = 0;
   int nflags = 0;                 // point-to-point flags in the control block (kernels/bert.cu)
   // workspace layout (byte offsets from the workspace base)

@@ -458,9 +458,12 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
     g.stages = g.BN == 256 ? 4 : g.BN == 128 ? 6 : 8;
     const int tiles = (int)(N / g.BN * mt);
     g.splits = 1;
-    if (tiles * 2 <= nsm)
-      for (int sp2 = 16; sp2 >= 2; sp2 >>= 1)
-        if (nk % sp2 == 0 && tiles * sp2 <= nsm) { g.splits = sp2; break; }
+    // split K only when a CTA would otherwise stream more than ~256 KB of operands: the split's
+    // partial round trip through L2 costs a few microseconds of latency
+    for (int sp2 = 1; sp2 <= 16 && nk % sp2 == 0 && tiles * sp2 <= nsm; sp2 *= 2) {
+      g.splits = sp2;
+      if ((128 + g.BN) * 2 * K / sp2 <= 256 * 1024) break;
+    }
     g.part = (float*)(base + sp.o_part);
     g.cnt = (unsigned*)(base + sp.o_cnt);
     op.grid = g.splits > 1 ? tiles * g.splits : std::min(tiles, nsm);

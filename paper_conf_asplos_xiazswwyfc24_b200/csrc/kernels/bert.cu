@@ -42,6 +42,7 @@ struct Ctrl {
   uint64_t afull[BA_SLOTS];
   uint64_t aempty[BA_SLOTS];
   uint64_t accb;
+  uint64_t recvb;               // cluster-pair split-K: the partner's half tile has landed
   uint64_t attb;
   uint64_t qkvb;
   uint32_t tmem_base;
@@ -205,7 +206,7 @@ __device__ void weight_producer(const BertParams& P, Ctrl* C, char* wring) {
 struct MmaState {
   uint32_t wit;            // weight-ring consumer group counter (thread 0)
   uint32_t aload, ause;    // A-ring chunk counters (thread 0)
-  uint32_t accph, attph, qkvph;
+  uint32_t accph, attph, qkvph, recvph;
 };
 
 // Epilogue of one 128 x nt accumulator tile, straight from registers: warp w reads TMEM lanes
@@ -308,6 +309,84 @@ __device__ __forceinline__ void tail_bias(const BertParams& P, const BStage& st,
   }
 }
 
+// Cluster-pair split-K (st.cpair): the two CTAs of a cluster computed the two K halves of the same
+// 128 x (4 HC) tile.  CTA rank r finalises columns [2 HC r, 2 HC r + 2 HC): it sends the partner's
+// columns of its partial into the partner's shared memory (one DSMEM bulk copy), then
+// adds the partner's contribution to its own half and runs the fused epilogue on HC columns per warp
+// half.  The A bytes each CTA streams are halved (K / 2) for one 8-16 KB exchange.
+template <int HC>
+__device__ __forceinline__ void pair_tail(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0,
+                                          char* recv, char* stage) {
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int q = warp & 3, half = warp >> 2, row = q * 32 + lane;
+  const uint32_t rank = (uint32_t)blockIdx.x & 1u;   // == split == cluster rank
+  const int c0 = n0 + (int)rank * 2 * HC + half * HC;
+  float4 bq[HC / 4];
+#pragma unroll
+  for (int c = 0; c < HC; c += 4) bq[c / 4] = __ldg(reinterpret_cast<const float4*>(st.bias + c0 + c));
+  ptx::mbar_wait(&C->accb, ms.accph);
+  ms.accph ^= 1;
+  ptx::tc_fence_after();
+  if (tid == 0) submark(P, st, 3);
+  const uint32_t lanes = C->tmem_base + ((uint32_t)(q * 32) << 16);
+  constexpr uint32_t kBytes = 128 * 2 * HC * 4;
+  if (tid == 0) ptx::mbar_arrive_expect_tx(&C->recvb, kBytes);   // the partner's half tile, by bulk copy
+  float v[HC];
+  // ---- the partner's columns of this partial -> local staging (the A ring: its MMAs completed), then
+  // one bulk DSMEM copy into the partner's receive buffer, completing on the partner's mbarrier
+  if constexpr (HC == 8) ptx::tmem_ld8(lanes + (rank ^ 1u) * 2 * HC + half * HC, v);
+  else ptx::tmem_ld16(lanes + (rank ^ 1u) * 2 * HC + half * HC, v);
+  float* stg = reinterpret_cast<float*>(stage) + row * 2 * HC + half * HC;
+#pragma unroll
+  for (int c = 0; c < HC; c += 4) *reinterpret_cast<float4*>(stg + c) = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
+  // ---- own columns
+  if constexpr (HC == 8) ptx::tmem_ld8(lanes + rank * 2 * HC + half * HC, v);
+  else ptx::tmem_ld16(lanes + rank * 2 * HC + half * HC, v);
+  ptx::tc_fence_before();
+  ptx::fence_proxy_async_smem();   // generic smem writes -> the async-proxy bulk copy
+  csync();
+  if (tid == 0)
+    ptx::bulk_s2cluster(ptx::mapa(ptx::smem_u32(recv), rank ^ 1u), stage, kBytes,
+                        ptx::mapa(ptx::smem_u32(&C->recvb), rank ^ 1u));
+  // the staging area is next written by a TMA load of a later stage, which comes after a grid
+  // barrier that the partner only reaches once this copy has completed on its mbarrier
+  ptx::mbar_wait(&C->recvb, ms.recvph);
+  ms.recvph ^= 1;
+  if (tid == 0) submark(P, st, 8);
+  if (row >= P.S) return;
+  const float* rp = reinterpret_cast<const float*>(recv) + row * 2 * HC + half * HC;
+#pragma unroll
+  for (int c = 0; c < HC; c += 4) {
+    const float4 o = *reinterpret_cast<const float4*>(rp + c);
+    const float4 b = bq[c / 4];
+    v[c] += o.x + b.x; v[c + 1] += o.y + b.y; v[c + 2] += o.z + b.z; v[c + 3] += o.w + b.w;
+  }
+  const int S = P.S, N = st.N;
+  if (st.epi == EP_GELU) {
+#pragma unroll
+    for (int c = 0; c < HC; ++c) v[c] = gelu_erf(v[c]);
+    uint4* dst = reinterpret_cast<uint4*>(st.out_b + (int64_t)row * N + c0);
+#pragma unroll
+    for (int c = 0; c < HC; c += 8)
+      dst[c / 8] = make_uint4(pack_bf16(v[c], v[c + 1]), pack_bf16(v[c + 2], v[c + 3]), pack_bf16(v[c + 4], v[c + 5]),
+                              pack_bf16(v[c + 6], v[c + 7]));
+    return;
+  }
+  const int H = N / 3;   // EP_QKV (HC columns inside one head)
+  const int which = c0 / H, hh = (c0 % H) >> 6, jd = c0 & 63;
+  if (which < 2) {
+    uint4* dst = reinterpret_cast<uint4*>(st.out_b + (((int64_t)(which * st.heads + hh) * S + row) << 6) + jd);
+#pragma unroll
+    for (int c = 0; c < HC; c += 8)
+      dst[c / 8] = make_uint4(pack_bf16(v[c], v[c + 1]), pack_bf16(v[c + 2], v[c + 3]), pack_bf16(v[c + 4], v[c + 5]),
+                              pack_bf16(v[c + 6], v[c + 7]));
+  } else {
+    uint16_t* dst = st.out_vt + ((int64_t)hh * 64 + jd) * S + row;
+#pragma unroll
+    for (int c = 0; c < HC; ++c) dst[(int64_t)c * S] = bf16_bits(v[c]);
+  }
+}
+
 template <int COLS>
 __device__ __forceinline__ void gemm_tail(const BertParams& P, const BStage& st, Ctrl* C, MmaState& ms, int n0,
                                           int split, char* areg) {
@@ -375,6 +454,13 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
   }
 
   // ---- epilogue (all 8 warps: warp w reads TMEM lanes 32*(w%4).., column half w/4)
+  if (st.cpair) {
+    char* recv = areg + B_AREGION;
+    if (nt == 32) pair_tail<8>(P, st, C, ms, n0, recv, areg);
+    else pair_tail<16>(P, st, C, ms, n0, recv, areg);
+    if (tid == 0) submark(P, st, 4);
+    return;
+  }
   switch (nt) {
     case 16: gemm_tail<8>(P, st, C, ms, n0, split, areg); break;
     case 32: gemm_tail<16>(P, st, C, ms, n0, split, areg); break;
@@ -653,6 +739,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
       ptx::mbar_init(&C->aempty[i], 1);
     }
     ptx::mbar_init(&C->accb, 1);
+    ptx::mbar_init(&C->recvb, 1);
     ptx::mbar_init(&C->attb, 1);
     ptx::mbar_init(&C->qkvb, 1);
     ptx::fence_mbar_init();
@@ -661,6 +748,12 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
+  // the CTA pair (cluster) exchanges partial tiles through each other's shared memory: both CTAs
+  // must have started and initialised their mbarriers before either sends (cluster barrier)
+  if (P.pairs) {
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+  }
 
   if (warp == 8) {
     const int lane = tid & 31;
@@ -670,7 +763,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
   }
   // ---- stage executor (warps 0-7).  Stage descriptors are double-buffered in smem: stage s+1's is
   // fetched while stage s runs, so it is never on the critical path behind a grid barrier.
-  MmaState ms{0u, 0u, 0u, 0u, 0u, 0u};
+  MmaState ms{0u, 0u, 0u, 0u, 0u, 0u, 0u};
   if (tid < (int)(sizeof(BStage) / 16))
     reinterpret_cast<int4*>(sbuf + (P.s_begin & 1))[tid] = __ldg(reinterpret_cast<const int4*>(P.stages + P.s_begin) + tid);
   csync();
@@ -747,7 +840,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
 
 }  // namespace bert
 
-cudaError_t bert_launch(const BertParams& prm, int grid, cudaStream_t s) {
+cudaError_t bert_launch(const BertParams& prm, int grid, bool pairs, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(bert::bert_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, B_SMEM);
@@ -759,11 +852,15 @@ cudaError_t bert_launch(const BertParams& prm, int grid, cudaStream_t s) {
   cfg.blockDim = dim3(BERT_THREADS);
   cfg.dynamicSmemBytes = B_SMEM;
   cfg.stream = s;
-  cudaLaunchAttribute at[1];
+  cudaLaunchAttribute at[2];
   at[0].id = cudaLaunchAttributeCooperative;
   at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeClusterDimension;   // CTA pairs (cluster-pair split-K stages)
+  at[1].val.clusterDim.x = 2;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
   cfg.attrs = at;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = pairs ? 2 : 1;
   return cudaLaunchKernelEx(&cfg, bert::bert_kernel, prm);
 }
 

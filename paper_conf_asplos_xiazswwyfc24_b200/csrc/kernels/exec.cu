@@ -771,6 +771,16 @@ __device__ __noinline__ void run_reduce(const Params& P, const Stage& st, char* 
     const int64_t o = ob + sub;
     const bool live = o < st.rows;
     float acc = st.red_fn ? -INFINITY : 0.f;
+    // a mean (sum with scale 1/E) is accumulated relative to the row's first element v0 and
+    // returned as v0 + scale * sum(v - v0): exact for a constant row, no loss of the small spread
+    // of an offset row (the LayerNorm mean, then x - mean, must be exactly 0 for a constant row)
+    const bool shifted = st.red_fn == 0 && st.red_scale != 1.f;
+    float v0 = 0.f;
+    if (live && shifted) {
+      float z1[1] = {0.f}, d1[MAX_RED] = {0.f, 0.f, 0.f, 0.f}, e1[1];
+      run_prog<1>(P, pre, o, 0, 1, z1, d1, e1);
+      v0 = e1[0];
+    }
     if (live) {
       for (int64_t c0 = (int64_t)gl * CHUNK; c0 < st.cols; c0 += (int64_t)G * CHUNK) {
         int nv = (int)((st.cols - c0) < CHUNK ? (st.cols - c0) : CHUNK);
@@ -780,14 +790,14 @@ __device__ __noinline__ void run_reduce(const Params& P, const Stage& st, char* 
         run_prog<CHUNK>(P, pre, o, c0, nv, zero, dummy, vals);
 #pragma unroll
         for (int j = 0; j < CHUNK; ++j)
-          if (j < nv) acc = st.red_fn ? fmaxf(acc, vals[j]) : acc + vals[j];
+          if (j < nv) acc = st.red_fn ? fmaxf(acc, vals[j]) : acc + (vals[j] - v0);
       }
     }
     for (int s2 = G >> 1; s2 > 0; s2 >>= 1) {
       float y = __shfl_xor_sync(0xffffffffu, acc, s2);
       acc = st.red_fn ? fmaxf(acc, y) : acc + y;
     }
-    acc *= st.red_scale;
+    acc = shifted ? v0 + acc * st.red_scale : acc * st.red_scale;
     if (live && gl == 0) {
       float a1[1] = {acc};
       run_prog<1>(P, post, o, 0, 1, a1, red);

@@ -226,11 +226,11 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       ptx::tc_fence_before();
       ptx::mbar_arrive(&C->tempty[buf]);
       if (SP > 1) {
-        // meet the other splits of this tile (all units are co-resident: grid == units <= #SMs)
-        __threadfence();
+        // meet the other splits of this tile (all units are co-resident: grid == units <= #SMs);
+        // the barrier orders every epilogue thread's partial stores before thread et == 0's release
         epi_sync();
         if (et == 0) {
-          atomicAdd(&g.cnt[t], 1u);
+          ptx::red_release_add(&g.cnt[t], 1u);
           while (ptx::ld_acquire(&g.cnt[t]) < (unsigned)SP) {
           }
         }
@@ -471,18 +471,24 @@ __global__ void sw_bias_kernel(const SwBias B) {
   pdl_wait();
   trace_stamp(B.trace, B.op);
   const SwBiasEnt& E = B.ent[blockIdx.y];
-  const int L2 = B.L2;
-  const int64_t n = (int64_t)E.nW * E.heads * SW_TAB;
+  const int L2 = B.L2, L22 = L2 * L2;
+  constexpr int G = SW_TAB / 4;   // float4 groups per (window, head) tile
+  const int64_t n = (int64_t)E.nW * E.heads * G;
   for (int64_t o = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; o < n; o += (int64_t)gridDim.x * blockDim.x) {
-    const int t = (int)(o % SW_TAB);
-    const int64_t u = o / SW_TAB;           // (w, h) unit of the table
+    const int g = (int)(o % G);
+    const int64_t u = o / G;           // (w, h) unit of the table
     const int h = (int)(u % E.heads), w = (int)(u / E.heads);
-    float v = 0.f;
-    if (t < L2 * L2) {
-      v = __ldg(E.bias + (int64_t)h * L2 * L2 + t);
-      if (E.mask) v += __ldg(E.mask + (int64_t)w * L2 * L2 + t);
+    float v[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int t = 4 * g + e;
+      v[e] = 0.f;
+      if (t < L22) {
+        v[e] = __ldg(E.bias + (int64_t)h * L22 + t);
+        if (E.mask) v[e] += __ldg(E.mask + (int64_t)w * L22 + t);
+      }
     }
-    E.dst[o] = v;
+    reinterpret_cast<float4*>(E.dst)[o] = make_float4(v[0], v[1], v[2], v[3]);
   }
 }
 
@@ -525,15 +531,19 @@ __global__ void __launch_bounds__(256) sw_pool_kernel(const SwHead H) {
     const float* xr = H.x + ((int64_t)b * H.L + t) * C;
     float4 v[8];
     float m = 0.f;
-    for (int k = 0; k < NV; ++k) {
-      v[k] = __ldg(reinterpret_cast<const float4*>(xr) + lane + 32 * k);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      v[k] = k < NV ? __ldg(reinterpret_cast<const float4*>(xr) + lane + 32 * k) : make_float4(0.f, 0.f, 0.f, 0.f);
       m += (v[k].x + v[k].y) + (v[k].z + v[k].w);
     }
     m *= 1.f / (float)(4 * NV);
     float M2 = 0.f, n = (float)(4 * NV);
-    for (int k = 0; k < NV; ++k) {
-      const float a = v[k].x - m, bb = v[k].y - m, c = v[k].z - m, d = v[k].w - m;
-      M2 += (a * a + bb * bb) + (c * c + d * d);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (k < NV) {
+        const float a = v[k].x - m, bb = v[k].y - m, c = v[k].z - m, d = v[k].w - m;
+        M2 += (a * a + bb * bb) + (c * c + d * d);
+      }
     }
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -544,7 +554,9 @@ __global__ void __launch_bounds__(256) sw_pool_kernel(const SwHead H) {
       n *= 2.f;
     }
     const float rs = rsqrtf(M2 / (float)C + H.eps);
-    for (int k = 0; k < NV; ++k) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      if (k >= NV) break;
       const int e = 4 * (lane + 32 * k);
       const float4 gm = __ldg(reinterpret_cast<const float4*>(H.gamma + e));
       const float4 bt = __ldg(reinterpret_cast<const float4*>(H.beta + e));
@@ -682,7 +694,8 @@ cudaError_t sw_launch_row(const SwRow& r, cudaStream_t s) {
 }
 
 cudaError_t sw_launch_bias(const SwBias& b, int max_table, cudaStream_t s) {
-  return launch_pdl(swin::sw_bias_kernel, dim3((unsigned)std::min(64, (max_table + 1023) / 1024), b.n), dim3(256), 0, s, b);
+  return launch_pdl(swin::sw_bias_kernel, dim3((unsigned)std::max(1, std::min(256, max_table / 4 / 256)), b.n), dim3(256), 0,
+                    s, b);
 }
 
 cudaError_t sw_launch_im2col(const SwIm2col& p, cudaStream_t s) {

@@ -169,3 +169,30 @@ def test_bound_bias_updated_in_place_is_seen(record_err):
     emu = te.evaluate(spec, og.bert_feed(X, plist, x, w), bf16_operands=True)[y]
     assert np.abs(out1 - out0).max() > 0.1
     record_err(float(np.abs(out1 - emu).max()), 2e-2)
+
+
+@pytest.mark.parametrize("kind", ["constant", "offset"])
+def test_layernorm_degenerate_rows_generic_executor(kind, record_err):
+    """The same LayerNorm pins on the generic fused executor (exec.cu, tiny fp32 BERT layer): the
+    reduction stage's mean is shifted by the row's first element, so a constant row normalises to
+    beta and an offset row keeps its noise (fp32 path tolerance: rel 1e-4 of max(|o|, rms))."""
+    cfg = dict(synth.BERT_TINY)
+    S, H = cfg["seq"], cfg["hidden"]
+    w = synth.bert_weights(cfg)
+    for k in ("Wo", "W2", "bo", "c2"):
+        w[0][k] = np.zeros_like(w[0][k])
+    if kind == "constant":
+        x = np.repeat((np.arange(S, dtype=np.float32) * 0.37 - 5.0)[:, None], H, axis=1).astype(np.float32)
+        x[::5] = 1000.0
+    else:
+        x = (1000.0 + synth.normal(92, (S, H))).astype(np.float32)
+    spec, X, plist, y = og.bert(cfg)
+    ref = te.evaluate(spec, og.bert_feed(X, plist, x, w))[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    plan = g.partition(L.device_query(0))
+    assert "pattern bert: not used" in plan.describe()
+    s = session(g, plan, og.bert_feed(gX, gpl, x, w), [gy])
+    s.run()
+    out = s.result(gy)
+    rms = np.sqrt(np.mean(ref ** 2))
+    record_err(float(np.max(np.abs(out - ref) / np.maximum(np.abs(ref), rms))), 1e-4, kind=kind)

@@ -1,0 +1,12 @@
+#!/bin/bash
+mkdir -p gpurun_out
+python -c "from paper_conf_asplos_xiazswwyfc24_b200.build import build; build()" > gpurun_out/build.log 2>&1
+timeout 600 python -m pytest tests/test_gpu_bert_stages.py tests/test_gpu_parity.py -q -x -m gpu -k "bert or stage or layernorm or bias" > gpurun_out/pytest_bert.txt 2>&1
+echo "rc=$?" >> gpurun_out/pytest_bert.txt
+for v in 1 0; do SOUFFLE_BERT_PAIRS=$v timeout 300 python tools/sweep_bert.py "" > gpurun_out/pairs_$v.txt 2>&1; done
+timeout 300 python tools/profile_bert.py 12 > gpurun_out/timeline.txt 2>&1
+timeout 300 python tools/graph_timing.py > gpurun_out/graph_timing.json 2> gpurun_out/graph_timing.err
+export PYTHONPATH=$PWD
+timeout 900 compute-sanitizer --tool racecheck --print-limit 10 python tools/san_case.py bert_small > gpurun_out/san_racecheck_bert.txt 2>&1
+python tools/swin_trace.py 1 > gpurun_out/trace_b1.txt 2>&1
+echo done

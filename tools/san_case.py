@@ -1,0 +1,42 @@
+"""One small launch of a kernel family, checked against the oracle (for compute-sanitizer runs).
+usage: python tools/san_case.py bert_small | swin_small | generic_tiny"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+import synth.swin as SW  # noqa: E402
+from oracle import graphs as og  # noqa: E402
+from oracle import te  # noqa: E402
+from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L  # noqa: E402
+from paper_conf_asplos_xiazswwyfc24_b200 import models as M  # noqa: E402
+from paper_conf_asplos_xiazswwyfc24_b200.session import session  # noqa: E402
+
+which = sys.argv[1]
+if which in ("bert_small", "generic_tiny"):
+    cfg = dict(synth.BERT_BASE, seq=32, hidden=256, heads=4, ffn=1024, layers=2) if which == "bert_small" else synth.BERT_TINY
+    x, w = synth.bert_input(cfg), synth.bert_weights(cfg)
+    spec, X, plist, y = og.bert(cfg)
+    ref = te.evaluate(spec, og.bert_feed(X, plist, x, w), bf16_operands=cfg["gemm_dtype"] == "bf16")[y]
+    g, gX, gpl, gy = M.bert(cfg)
+    plan = g.partition(L.device_query(0))
+    s = session(g, plan, og.bert_feed(gX, gpl, x, w), [gy])
+    s.run()
+    out = s.result(gy)
+else:
+    cfg = dict(SW.SWIN_TINY, embed=128, heads=(4, 8), gemm_dtype="bf16")
+    P = SW.swin_params(cfg)
+    fv = SW.swin_feed_values(cfg, P)
+    img = SW.swin_input(cfg)
+    g, names, gx, gy = M.swin(cfg)
+    feed = {names[k]: v for k, v in fv.items()}
+    feed[gx] = img
+    plan = g.partition(L.device_query(0))
+    s = session(g, plan, feed, [gy])
+    s.run()
+    out = s.result(gy)
+    spec, on, ox, oy = og.swin(cfg)
+    ref = te.evaluate(spec, feed, bf16_operands=True)[oy]
+print(which, plan.describe().splitlines()[0][:100], "max abs err", float(np.abs(out - ref).max()))
