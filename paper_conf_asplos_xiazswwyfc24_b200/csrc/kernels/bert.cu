@@ -525,22 +525,26 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
     const float c = st.scale * 1.4426950408889634f;
     float sv[64];
     ptx::tmem_ld64(tb, sv);
-    float mx = -INFINITY;
+    if (S < 128) {   // keys beyond S (TMA zero-fill)
 #pragma unroll
-    for (int j = 0; j < 64; ++j) {
-      if (half * 64 + j >= S) sv[j] = -INFINITY;   // keys beyond S (TMA zero-fill)
-      mx = fmaxf(mx, sv[j]);
+      for (int j = 0; j < 64; ++j)
+        if (half * 64 + j >= S) sv[j] = -INFINITY;
     }
+    float m4[4] = {sv[0], sv[1], sv[2], sv[3]};   // 4 independent chains (no 64-long dependency)
+#pragma unroll
+    for (int j = 4; j < 64; ++j) m4[j & 3] = fmaxf(m4[j & 3], sv[j]);
+    const float mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
     // each half normalises with its own max; one (max, sum) exchange combines the halves:
     // z = z_a 2^{(m_a - m)c} + z_b 2^{(m_b - m)c}, p_j = 2^{(s_j - m_a)c} 2^{(m_a - m)c} / z
     const float mxs = (mx == -INFINITY) ? 0.f : mx;   // a fully masked half contributes 0
     const float mc = mxs * c;
-    float z = 0.f;
+    float z4[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
     for (int j = 0; j < 64; ++j) {
       sv[j] = ptx::ex2(fmaf(sv[j], c, -mc));
-      z += sv[j];
+      z4[j & 3] += sv[j];
     }
+    const float z = (z4[0] + z4[1]) + (z4[2] + z4[3]);
     float2* xch = reinterpret_cast<float2*>(Qs);   // [2][128] (max, sum); Q is consumed (S complete)
     xch[half * 128 + row] = make_float2(mx, z);
     csync();
@@ -557,7 +561,7 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
     }
     ptx::tc_fence_before();
   }
-  ptx::fence_proxy_async();
+  ptx::fence_proxy_async_smem();   // P / ctx smem writes -> the MMA (async proxy)
   csync();
   if (tid == 0) submark(P, st, 3);
   // ---- O = P V  (M = 128, N = 64, K = 128 keys) -> TMEM columns [128, 192)
@@ -587,7 +591,7 @@ __device__ void run_attn(const BertParams& P, const BStage& st, Ctrl* C, char* w
                      pack_bf16(o[8 * j + 4], o[8 * j + 5]), pack_bf16(o[8 * j + 6], o[8 * j + 7]));
     ptx::tc_fence_before();
   }
-  ptx::fence_proxy_async();
+  ptx::fence_proxy_async_smem();   // P / ctx smem writes -> the MMA (async proxy)
   csync();
   // ---- partial_h = ctx_h Wo[tile rows, h-slice]^T  (M = 128, N = nt, K = 64) -> TMEM columns [0, nt)
   if (warp == 0) {
