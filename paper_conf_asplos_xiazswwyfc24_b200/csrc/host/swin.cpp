@@ -459,10 +459,12 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
     const int tiles = (int)(N / g.BN * mt);
     g.splits = 1;
     // split K only when a CTA would otherwise stream more than ~256 KB of operands: the split's
-    // partial round trip through L2 costs a few microseconds of latency
+    // partial round trip through L2 costs a few microseconds of latency.  Residual epilogues add
+    // their partials with atomics (no round trip), so they split down to ~96 KB per CTA
+    const int64_t cap = epi == SWE_RESID ? 96 * 1024 : 256 * 1024;
     for (int sp2 = 1; sp2 <= 16 && nk % sp2 == 0 && tiles * sp2 <= nsm; sp2 *= 2) {
       g.splits = sp2;
-      if ((128 + g.BN) * 2 * K / sp2 <= 256 * 1024) break;
+      if ((128 + g.BN) * 2 * K / sp2 <= cap) break;
     }
     g.part = (float*)(base + sp.o_part);
     g.cnt = (unsigned*)(base + sp.o_cnt);

@@ -217,6 +217,27 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
         ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
         if (SP == 1) {
           if (r < g.M) epi_chunk(g, r, n0 + c0, v);
+        } else if (g.epi == SWE_RESID) {
+          // residual epilogue is linear: every split adds its partial (split 0 also the bias)
+          // straight into the fp32 residual stream with vector atomics -- no partial round trip
+          // (the order of the fp32 adds varies from run to run: ulp-level nondeterminism)
+          if (r < g.M) {
+            if (split == 0 && g.bias) {
+              const float4* bp = reinterpret_cast<const float4*>(g.bias + n0 + c0);
+#pragma unroll
+              for (int c = 0; c < 32; c += 4) {
+                const float4 b = __ldg(bp + c / 4);
+                v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
+              }
+            }
+            const int tok = g.rowmap ? __ldg(g.rowmap + r) : r;
+            float* xp = g.out_f + (int64_t)tok * g.N + n0 + c0;
+#pragma unroll
+            for (int c = 0; c < 32; c += 4)
+              asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(xp + c), "f"(v[c]), "f"(v[c + 1]),
+                           "f"(v[c + 2]), "f"(v[c + 3])
+                           : "memory");
+          }
         } else {   // fp32 partial of this split
           float4* dst = reinterpret_cast<float4*>(g.part + ((int64_t)u * 128 + rt) * BN + c0);
 #pragma unroll
@@ -225,7 +246,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       }
       ptx::tc_fence_before();
       ptx::mbar_arrive(&C->tempty[buf]);
-      if (SP > 1) {
+      if (SP > 1 && g.epi != SWE_RESID) {
         // meet the other splits of this tile (all units are co-resident: grid == units <= #SMs);
         // the barrier orders every epilogue thread's partial stores before thread et == 0's release
         epi_sync();

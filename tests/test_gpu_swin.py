@@ -66,7 +66,8 @@ def test_swin_pattern_small(batch, record_err):
     got, again, ref, plan = _run(dict(SWIN_PAT, batch=batch), bf16=True)
     assert "pattern swin: batch" in plan.describe()
     record_err(float(np.max(np.abs(got - ref))), 2e-2, batch=batch, rms=float(np.sqrt(np.mean(ref ** 2))))
-    assert np.array_equal(got, again)          # no atomics on the data path: bit-reproducible
+    # split-K residual epilogues accumulate with fp32 atomics: repeat runs agree to fp32 rounding
+    assert np.max(np.abs(got - again)) <= 1e-5 * max(1.0, float(np.max(np.abs(got))))
 
 
 def test_swin_pattern_generic_agree():
