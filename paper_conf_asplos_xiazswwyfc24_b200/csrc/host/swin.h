@@ -33,6 +33,7 @@ struct SwinOp {
   SwHead head{};
   SwBias bias{};
   int grid = 0;
+  bool two_sm = false;          // GEMM on CTA pairs (sw_gemm2_kernel, cta_group::2)
   // tensor map requests: (buffer id, rows, cols, box rows, box cols, swizzle bytes); buffer ids are
   // workspace offsets (>= 0) or -(node + 1) for a bound tensor
   struct Map { int64_t buf; int64_t rows, cols; int box_rows, box_cols, swz; };

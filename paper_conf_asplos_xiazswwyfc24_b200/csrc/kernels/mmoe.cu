@@ -72,15 +72,26 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   for (int k = tid; k < T; k += MMOE_THREADS) bo[k] = __ldg(P.bo[k]);
   __syncthreads();   // mbarrier initialised before anyone waits on it
   ptx::mbar_wait(&bar, 0);
-  // ---- 1: fused expert + gate GEMM, one warp per (row, batch) output, lanes split D
-  for (int o = warp; o < R * B; o += MMOE_THREADS / 32) {
-    const int r = o % R, b = o / R;
-    float s = 0.f;
-    for (int k = lane; k < D; k += 32) s = fmaf(xs[b * D + k], wsm(W1, (int64_t)r * D + k, f32), s);
+  // ---- 1: fused expert + gate GEMM; a warp computes 4 (row, batch) outputs at once (lanes split D,
+  // four independent accumulators and shuffle trees in flight: the chain latency is paid once per 4)
+  constexpr int kO = 4, kWarps = MMOE_THREADS / 32;
+  for (int o0 = warp * kO; o0 < R * B; o0 += kWarps * kO) {
+    float s[kO] = {0.f, 0.f, 0.f, 0.f};
+    for (int k = lane; k < D; k += 32) {
 #pragma unroll
-    for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-    if (lane == 0) {
-      const float v = s + b1[r];
+      for (int j = 0; j < kO; ++j) {
+        const int o = o0 + j;
+        if (o < R * B) s[j] = fmaf(xs[(o / R) * D + k], wsm(W1, (int64_t)(o % R) * D + k, f32), s[j]);
+      }
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1)
+#pragma unroll
+      for (int j = 0; j < kO; ++j) s[j] += __shfl_xor_sync(0xffffffffu, s[j], off);
+    if (lane < kO && o0 + lane < R * B) {
+      const int o = o0 + lane, r = o % R, b = o / R;
+      const float sl = lane == 0 ? s[0] : lane == 1 ? s[1] : lane == 2 ? s[2] : s[3];
+      const float v = sl + b1[r];
       o1[b * R + r] = r < E * De ? fmaxf(v, 0.f) : v;
     }
   }

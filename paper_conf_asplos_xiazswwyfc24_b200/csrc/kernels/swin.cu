@@ -56,7 +56,9 @@ __device__ __forceinline__ void trace_stamp(unsigned long long* tr, int op) {
     tr[op] = t;
   }
 }
-__device__ __forceinline__ void epi_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+constexpr int kEpiWarps = SW_GEMM_THREADS / 32 - 2, kEpiThreads = 32 * kEpiWarps, kEpiGroups = kEpiWarps / 4;
+static_assert(kEpiWarps % 4 == 0, "epilogue warps cover the 4 TMEM lane quarters evenly");
+__device__ __forceinline__ void epi_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kEpiThreads) : "memory"); }
 
 // K-major operand tile with 64-byte swizzle (rows of 32 bf16): 8-row groups 512 B apart
 __device__ __forceinline__ uint64_t sdesc_sw64(uint32_t saddr) {
@@ -71,8 +73,21 @@ __device__ __forceinline__ uint64_t sdesc_sw64(uint32_t saddr) {
 
 // ================================================================== GEMM
 // 32 consecutive accumulator columns [n, n + 32) of row r (r < M) through the fused epilogue
-__device__ __forceinline__ void epi_chunk(const SwGemm& g, int r, int n, float* v) {
-  if (g.bias) {
+// the chunk's bias, loaded before its accumulator columns are read from TMEM (the loads are in flight
+// during the tcgen05.ld instead of stalling the epilogue after it)
+__device__ __forceinline__ void bias_chunk(const SwGemm& g, int n, float4* b) {
+#pragma unroll
+  for (int c = 0; c < 8; ++c) b[c] = g.bias ? __ldg(reinterpret_cast<const float4*>(g.bias + n) + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
+__device__ __forceinline__ void epi_chunk(const SwGemm& g, int r, int n, float* v, const float4* bq = nullptr) {
+  if (bq) {
+#pragma unroll
+    for (int c = 0; c < 32; c += 4) {
+      const float4 b = bq[c / 4];
+      v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
+    }
+  } else if (g.bias) {
     const float4* bp = reinterpret_cast<const float4*>(g.bias + n);
 #pragma unroll
     for (int c = 0; c < 32; c += 4) {
@@ -142,7 +157,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
     }
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&C->tfull[i], 1);
-      ptx::mbar_init(&C->tempty[i], 256);
+      ptx::mbar_init(&C->tempty[i], kEpiThreads);
     }
     ptx::fence_mbar_init();
   }
@@ -201,8 +216,8 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       }
     }
   } else {
-    // ---- epilogue warps 2-9: warp w reads TMEM lanes 32 * (w % 4) .. (its lane quarter); the two
-    // warps of a quarter take alternate 32-column chunks
+    // ---- epilogue warps 2..: warp w reads TMEM lanes 32 * (w % 4) .. (its lane quarter); the
+    // kEpiGroups warps of a quarter take interleaved 32-column chunks
     const int q = warp & 3, eh = (warp - 2) >> 2, et = threadIdx.x - 64;
     uint32_t lt = 0;
     for (int u = blockIdx.x; u < units; u += gridDim.x, ++lt) {
@@ -212,11 +227,13 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       ptx::mbar_wait(&C->tfull[buf], use & 1);
       ptx::tc_fence_after();
       const int rt = q * 32 + lane, r = m0 + rt;
-      for (int c0 = 32 * eh; c0 < BN; c0 += 64) {
+      for (int c0 = 32 * eh; c0 < BN; c0 += 32 * kEpiGroups) {
         float v[32];
+        float4 bq[8];
+        if (SP == 1) bias_chunk(g, n0 + c0, bq);
         ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
         if (SP == 1) {
-          if (r < g.M) epi_chunk(g, r, n0 + c0, v);
+          if (r < g.M) epi_chunk(g, r, n0 + c0, v, bq);
         } else if (g.epi == SWE_RESID) {
           // residual epilogue is linear: every split adds its partial (split 0 also the bias)
           // straight into the fp32 residual stream with vector atomics -- no partial round trip
@@ -258,7 +275,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
         epi_sync();
         // reduce rows [split * 128 / SP, ...) of the tile, splits summed in order
         const int rows = 128 / SP, cpr = BN / 32;
-        for (int item = et; item < rows * cpr; item += 256) {
+        for (int item = et; item < rows * cpr; item += kEpiThreads) {
           const int rr = split * rows + item / cpr, c0 = (item % cpr) * 32;
           float v[32];
 #pragma unroll
@@ -286,6 +303,172 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
   ptx::tc_fence_before();
   __syncthreads();
   if (warp == 1) ptx::tmem_dealloc(tmem, (uint32_t)(2 * BN));
+}
+
+// ================================================================== 2-SM GEMM (cta_group::2)
+// For large M (batch >= 8): a CTA pair (cluster of 2, one TPC) computes a 256 x 256 tile with
+// tcgen05.mma.cta_group::2 -- each CTA loads its 128 rows of A and HALF of the 256 W rows, the tensor
+// cores of the pair read both halves, so every SM ingests 32 KB per 64-deep K chunk instead of 48 KB
+// for the same MMA work (the 1-SM 128 x 256 tile is bound by per-SM operand ingest).  Both CTAs'
+// TMA loads complete on the leader's barrier (.cta_group::2); rank 0 issues the MMAs; MMA completion
+// is multicast to both CTAs' barriers; each CTA's epilogue drains its own 128 TMEM lanes.
+struct Gemm2Ctrl {
+  uint64_t full[8], empty[8], tfull[2], tempty[2];
+  uint32_t tmem;
+};
+// TMA load into this CTA's shared memory whose completion is counted on an mbarrier of either CTA of
+// the pair (`bar`: shared::cluster address)
+__device__ __forceinline__ void tma2_load_2d(void* dst, const void* tmap, uint32_t bar, int32_t c0, int32_t c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          ptx::smem_u32(dst)),
+      "l"(tmap), "r"(bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+
+__device__ __forceinline__ void mma2_bf16_k64(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                              uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .b64 a1, a2, a3, b1, b2, b3;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "setp.eq.b32 q, 0, 0;\n\t"
+      "add.s64 a1, %1, 2;\n\tadd.s64 a2, %1, 4;\n\tadd.s64 a3, %1, 6;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], a1, b1, %3, q;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], a2, b2, %3, q;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], a3, b3, %3, q;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// MMA completion -> the same mbarrier offset in both CTAs of the pair
+__device__ __forceinline__ void mma2_commit_both(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                   ptx::smem_u32(bar)),
+               "h"((uint16_t)3)
+               : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+  asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+__global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm2_kernel(const __grid_constant__ GemmArgs A) {
+  extern __shared__ __align__(1024) char smem_raw[];
+  char* smem = (char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  Gemm2Ctrl* C = reinterpret_cast<Gemm2Ctrl*>(smem);
+  char* ring = smem + 1024;
+  const SwGemm& g = A.g;
+  constexpr int BN = 256;                     // pair tile: 256 rows x 256 columns
+  constexpr uint32_t A_BYTES = 16384, B_BYTES = 16384, STAGE = A_BYTES + B_BYTES;
+  const int NS = g.stages;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const int pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
+  const int ntn = g.N / BN, tiles = ntn * ((g.M + 255) / 256), nk = g.K / 64;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  pdl_trigger();
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) {
+      ptx::mbar_init(&C->full[i], 1);
+      ptx::mbar_init(&C->empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&C->tfull[i], 1);
+      ptx::mbar_init(&C->tempty[i], 2 * kEpiThreads);   // both CTAs' epilogue threads (leader's copy)
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 0 && lane == 0) {
+    ptx::prefetch_tmap(&A.ta);
+    ptx::prefetch_tmap(&A.tb);
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(ptx::smem_u32(&C->tmem)),
+                 "r"(2u * BN)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  cluster_sync_all();   // both CTAs' barriers initialised before any remote arrive / multicast commit
+  ptx::tc_fence_after();
+  const uint32_t tmem = C->tmem;
+  pdl_wait();
+  trace_stamp(g.trace, g.op);
+  const uint32_t leader_tempty[2] = {ptx::mapa(ptx::smem_u32(&C->tempty[0]), 0u), ptx::mapa(ptx::smem_u32(&C->tempty[1]), 0u)};
+
+  if (warp == 0) {
+    // ---- TMA producer: this CTA's 128 rows of A and its half (128 rows) of the 256 W rows; both
+    // CTAs' loads complete on the LEADER's full barrier (.cta_group::2), which expects both halves
+    const uint32_t full0 = ptx::mapa(ptx::smem_u32(&C->full[0]), 0u);
+    uint32_t it = 0;
+    for (int t = pair; t < tiles; t += npairs) {
+      const int m0 = (t / ntn) * 256 + (int)rank * 128, n0 = (t % ntn) * BN + (int)rank * 128;
+      for (int kc = 0; kc < nk; ++kc, ++it) {
+        const uint32_t slot = it % NS, ph = (it / NS) & 1;
+        ptx::mbar_wait(&C->empty[slot], ph ^ 1);
+        if (ptx::elect_one()) {
+          char* st = ring + slot * STAGE;
+          const uint32_t bar = full0 + slot * 8;
+          if (rank == 0) ptx::mbar_arrive_expect_tx(&C->full[slot], 2 * STAGE);
+          tma2_load_2d(st, &A.ta, bar, kc * 64, m0);
+          tma2_load_2d(st + A_BYTES, &A.tb, bar, kc * 64, n0);
+        }
+        __syncwarp();
+      }
+    }
+  } else if (warp == 1) {
+    uint32_t it = 0, lt = 0;
+    if (rank == 0) {
+      // ---- leader: MMA issue (M = 256 across the pair, N = 256, K = 16)
+      const uint32_t idesc = ptx::idesc_bf16(256, BN);
+      const uint64_t d0 = ptx::sdesc_sw128(ptx::smem_u32(ring));
+      for (int t = pair; t < tiles; t += npairs, ++lt) {
+        const uint32_t buf = lt & 1, use = lt >> 1;
+        ptx::mbar_wait_cluster(&C->tempty[buf], (use & 1) ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t d = tmem + buf * BN;
+        for (int kc = 0; kc < nk; ++kc, ++it) {
+          const uint32_t slot = it % NS, ph = (it / NS) & 1;
+          ptx::mbar_wait(&C->full[slot], ph);
+          ptx::tc_fence_after();
+          const uint64_t da = d0 + (uint64_t)((slot * STAGE) >> 4);
+          const uint64_t db = da + (uint64_t)(A_BYTES >> 4);
+          if (ptx::elect_one()) {
+            mma2_bf16_k64(d, da, db, idesc, kc > 0 ? 1u : 0u);
+            mma2_commit_both(&C->empty[slot]);
+            if (kc == nk - 1) mma2_commit_both(&C->tfull[buf]);
+          }
+          __syncwarp();
+        }
+      }
+    }
+  } else {
+    // ---- epilogue: this CTA's 128 rows of the pair tile (its own TMEM lanes)
+    const int q = warp & 3, eh = (warp - 2) >> 2;
+    uint32_t lt = 0;
+    for (int t = pair; t < tiles; t += npairs, ++lt) {
+      const uint32_t buf = lt & 1, use = lt >> 1;
+      const int m0 = (t / ntn) * 256 + (int)rank * 128, n0 = (t % ntn) * BN;
+      ptx::mbar_wait(&C->tfull[buf], use & 1);
+      ptx::tc_fence_after();
+      const int r = m0 + q * 32 + lane;
+      for (int c0 = 32 * eh; c0 < BN; c0 += 32 * kEpiGroups) {
+        float v[32];
+        float4 bq[8];
+        bias_chunk(g, n0 + c0, bq);
+        ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
+        if (r < g.M) epi_chunk(g, r, n0 + c0, v, bq);
+      }
+      ptx::tc_fence_before();
+      ptx::mbar_arrive_remote(leader_tempty[buf]);   // the leader's MMA reuses this buffer
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  cluster_sync_all();   // the peer's TMEM / smem are not released while the pair still uses them
+  if (warp == 1)
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(2u * BN) : "memory");
 }
 
 // ================================================================== window attention
@@ -688,6 +871,30 @@ cudaError_t sw_launch_gemm(const void* ta, const void* tb, const SwGemm& g, int 
   cudaError_t e = set_smem((const void*)swin::sw_gemm_kernel, 227 * 1024);
   if (e != cudaSuccess) return e;
   return launch_pdl(swin::sw_gemm_kernel, dim3(grid), dim3(SW_GEMM_THREADS), (size_t)sw_gemm_smem(g.BN, g.stages), s, a);
+}
+
+cudaError_t sw_launch_gemm2(const void* ta, const void* tb, const SwGemm& g, int grid, cudaStream_t s) {
+  swin::GemmArgs a;
+  memcpy(&a.ta, ta, sizeof(CUtensorMap));
+  memcpy(&a.tb, tb, sizeof(CUtensorMap));
+  a.g = g;
+  cudaError_t e = set_smem((const void*)swin::sw_gemm2_kernel, 227 * 1024);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(SW_GEMM_THREADS);
+  cfg.dynamicSmemBytes = (size_t)sw_gemm_smem(128, g.stages);   // 32 KB stages
+  cfg.stream = s;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  at[1].id = cudaLaunchAttributeClusterDimension;
+  at[1].val.clusterDim.x = 2;
+  at[1].val.clusterDim.y = 1;
+  at[1].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 2;
+  return cudaLaunchKernelEx(&cfg, swin::sw_gemm2_kernel, a);
 }
 
 cudaError_t sw_launch_attn(const void* tq, const void* tk, const void* tv, const SwAttn& at, int grid, cudaStream_t s) {

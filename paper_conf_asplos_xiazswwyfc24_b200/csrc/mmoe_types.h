@@ -6,7 +6,7 @@
 
 namespace souffle {
 
-enum { MMOE_THREADS = 256, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
+enum { MMOE_THREADS = 1024, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
 
 struct MmoeParams {
   const float* x;                  // [B][D]

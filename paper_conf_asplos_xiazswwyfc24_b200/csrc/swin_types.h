@@ -24,7 +24,8 @@ enum SwEpi : int32_t { SWE_F32 = 0, SWE_GELU = 1, SWE_RESID = 2, SWE_QKV = 3 };
 
 enum {
   SW_GEMM_THREADS = 320,      // warp 0 TMA producer, warp 1 MMA issuer, warps 2-9 epilogue (2 per
-                              // TMEM lane quarter, alternating 32-column chunks)
+                              // TMEM lane quarter, interleaved 32-column chunks; 12 epilogue warps
+                              // measured slower: register cap 128 -> spills)
   SW_ATTN_THREADS = 128,      // one thread per row of the M = 128 tile (two 64-row units)
   SW_ROW_THREADS = 256,       // 8 warps, one token row per warp
   SW_WIN_ROWS = 64,           // a (window, head) unit: 49 tokens padded to 64 rows

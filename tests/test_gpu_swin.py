@@ -66,8 +66,9 @@ def test_swin_pattern_small(batch, record_err):
     got, again, ref, plan = _run(dict(SWIN_PAT, batch=batch), bf16=True)
     assert "pattern swin: batch" in plan.describe()
     record_err(float(np.max(np.abs(got - ref))), 2e-2, batch=batch, rms=float(np.sqrt(np.mean(ref ** 2))))
-    # split-K residual epilogues accumulate with fp32 atomics: repeat runs agree to fp32 rounding
-    assert np.max(np.abs(got - again)) <= 1e-5 * max(1.0, float(np.max(np.abs(got))))
+    # split-K residual epilogues accumulate with fp32 atomics (order varies run to run): an ulp-level
+    # difference can flip a later bf16 operand rounding, so repeat runs agree to a few bf16 ulps
+    assert np.max(np.abs(got - again)) <= 5e-3
 
 
 def test_swin_pattern_generic_agree():
@@ -102,3 +103,44 @@ def test_swin_b_full_size(batch, record_err):
     assert (int(b), int(n)) == (batch, 1000) and pat == "True"
     assert float(e2) <= 2e-2
     record_err(float(e1), 2e-2, batch=batch, rms=float(rms))
+
+
+def _swin_b64_child():
+    """Swin-B at batch 64 (the per-GPU batch of the bench's 64-image replica job, 2-SM GEMM tiles)
+    against the oracle on sampled images: every image is independent, so the oracle evaluates the
+    batch-1 program on images 0, 37 and 63 only."""
+    cfg = dict(S.SWIN_B, batch=64)
+    P = S.swin_params(cfg)
+    fv = S.swin_feed_values(cfg, P)
+    img = S.swin_input(cfg)
+    g, names, x, y = M.swin(cfg)
+    feed = {names[k]: v for k, v in fv.items()}
+    feed[x] = img
+    plan = g.partition(L.device_query(0))
+    s = session(g, plan, feed, [y])
+    s.run()
+    got = s.result(y)
+    c1 = dict(S.SWIN_B, batch=1)
+    spec, onames, ox, oy = og.swin(c1)
+    errs = []
+    for i in (0, 37, 63):
+        f1 = {onames[k]: v for k, v in S.swin_feed_values(c1, S.swin_params(c1)).items()}
+        f1[ox] = img[i:i + 1]
+        ref = te.evaluate(spec, f1, bf16_operands=True)[oy]
+        errs.append(float(np.max(np.abs(got[i] - ref[0]))))
+    print("RESULT", max(errs), "pattern swin: batch 64" in plan.describe())
+
+
+def test_swin_b_batch64_sampled(record_err):
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_swin as t; t._swin_b64_child()" % (
+        root, os.path.join(root, "tests"))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=900, cwd=root)
+    line = [ln for ln in r.stdout.splitlines() if ln.startswith("RESULT")]
+    assert line, r.stderr[-2000:]
+    _, err, pat = line[0].split()
+    assert pat == "True"
+    record_err(float(err), 2e-2, batch=64, sampled_images=[0, 37, 63])
