@@ -1,6 +1,7 @@
 // MMoE pattern: strict match of models.mmoe's TE program and launch of the fused kernel
 // (kernels/mmoe.cu).  PAPER.md Table 2, §6.1 (horizontal fusion of the expert and gate GEMMs),
 // Table 5 (one kernel).
+#include <cstdlib>
 #include <cstring>
 #include <sstream>
 #include <string>
@@ -122,6 +123,7 @@ void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
   if (!c.ok || c.i != N.size()) return no("not an MMoE program (towers)");
   if (g.outputs != mp.y) return no("outputs are not the task towers");
   if (mp.E > MMOE_MAX_E || mp.T > MMOE_MAX_T || mp.B > MMOE_MAX_B) return no("too many experts / tasks / rows");
+  if (mp.B * mp.T > MMOE_THREADS / 32 || mp.Th > 32) return no("batch x tasks > warps or tower width > 32");
   const int epv = mp.w_f32 ? 4 : 8;   // weight tensors are staged by bulk copies of 16-byte multiples
   if ((int64_t)mp.De * mp.D % epv || (int64_t)mp.E * mp.D % epv || (int64_t)mp.Th * mp.De % epv || mp.Th % epv)
     return no("weight tensor sizes must be multiples of 16 bytes");
@@ -164,6 +166,7 @@ souffle_status mmoe_run(Plan& p, void* ws, void* stream) {
   }
   prm.B = mp.B; prm.D = mp.D; prm.E = mp.E; prm.De = mp.De; prm.T = mp.T; prm.Th = mp.Th;
   prm.w_f32 = mp.w_f32;
+  prm.pad = std::getenv("SOUFFLE_MMOE_DEBUG") ? 1 : 0;   // debug: per-phase clock deltas (printf)
   for (int k = 0; k < mp.E; ++k)
     if ((uintptr_t)prm.We[k] & 15) return fail(SOUFFLE_E_INVALID_ARG, "MMoE weights must be 16-byte aligned");
   for (int k = 0; k < mp.T; ++k)

@@ -64,7 +64,26 @@ __device__ __forceinline__ uint16_t bf16_bits(float a) {
   __nv_bfloat16 b = __float2bfloat16_rn(a);
   return *reinterpret_cast<uint16_t*>(&b);
 }
-__device__ __forceinline__ float gelu_erf(float x) { return 0.5f * x * (1.f + erff(x * 0.70710678118654752f)); }
+// erf-GELU (the TE's exact-erf semantics) with erf(t) = 1 - 2^(t P7(t)) on t = |x| <= 3.92 (erf = 1 in
+// fp32 beyond): one polynomial, one MUFU.EX2, no branch (CUDA's erff takes two divergent polynomial
+// paths).  |erf error| <= 3e-7 absolute (fit in DESIGN.md R19), GELU within 5e-7 absolute -- far
+// below the bf16 rounding of the GELU output that follows.
+__device__ __forceinline__ float gelu_erf(float x) {
+  const float u = x * 0.70710678118654752f;
+  const float t = fminf(fabsf(u), 3.92f);
+  float p = -4.4602740672416985e-05f;
+  p = fmaf(p, t, 4.394397255964577e-04f);
+  p = fmaf(p, t, -1.4703732449561357e-03f);
+  p = fmaf(p, t, -8.046277216635644e-04f);
+  p = fmaf(p, t, 2.8278736397624016e-02f);
+  p = fmaf(p, t, -0.14849244058132172f);
+  p = fmaf(p, t, -0.9184142351150513f);
+  p = fmaf(p, t, -1.627908706665039f);
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(t * p));
+  const float e = copysignf(1.f - y, u);
+  return 0.5f * x * (1.f + e);
+}
 template <class T>
 __device__ __forceinline__ const void* ldgp(T* const* p) {
   return (const void*)__ldg(reinterpret_cast<const unsigned long long*>(p));

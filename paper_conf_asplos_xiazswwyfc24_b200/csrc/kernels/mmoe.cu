@@ -10,6 +10,7 @@
 //   2  g_k = softmax(G_k)                       (max-subtracted, per task)
 //   3  f_k = sum_e g_k[e] E_e                    (the slice * expert products and their sum chain)
 //   4  y_k = W_o,k relu(W_t,k f_k + b_t,k) + b_o,k
+#include <cstdio>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -39,7 +40,6 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   const bool f32 = P.w_f32 != 0;
   const int es = f32 ? 4 : 2;
   const int R = E * De + T * E;               // rows of the horizontally fused GEMM
-  __shared__ __align__(8) uint64_t bar;
   // raw (storage dtype) weights, staged by bulk copies: [R][D] experts then gates, [T][Th][De], [T][Th]
   char* W1 = smraw;
   char* Wt = W1 + (((int64_t)R * D * es + 15) & ~15);
@@ -52,62 +52,75 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   float* f = o1 + B * R;                      // [B][T][De]
   float* h1 = f + B * T * De;                 // [B][T][Th]
 
-  // ---- every weight tensor in flight at once: one bulk copy (TMA engine) per tensor, one mbarrier
-  if (tid == 0) {
-    ptx::mbar_init(&bar, 1);
-    ptx::fence_mbar_init();
-    const uint32_t bytes = (uint32_t)(((int64_t)E * De * D + (int64_t)T * E * D + (int64_t)T * Th * De + T * Th) * es);
-    ptx::mbar_arrive_expect_tx(&bar, bytes);
-    for (int e = 0; e < E; ++e)
-      ptx::bulk_g2s(W1 + (int64_t)e * De * D * es, P.We[e], (uint32_t)(De * D * es), &bar);
-    for (int k = 0; k < T; ++k)
-      ptx::bulk_g2s(W1 + (int64_t)(E * De + k * E) * D * es, P.Wg[k], (uint32_t)(E * D * es), &bar);
-    for (int k = 0; k < T; ++k) ptx::bulk_g2s(Wt + (int64_t)k * Th * De * es, P.Wt[k], (uint32_t)(Th * De * es), &bar);
-    for (int k = 0; k < T; ++k) ptx::bulk_g2s(Wo + (int64_t)k * Th * es, P.Wo[k], (uint32_t)(Th * es), &bar);
-  }
-  for (int i = tid; i < B * D; i += MMOE_THREADS) xs[i] = __ldg(P.x + i);
-  for (int r = tid; r < R; r += MMOE_THREADS)
-    b1[r] = r < E * De ? __ldg(P.be[r / De] + r % De) : __ldg(P.bg[(r - E * De) / E] + (r - E * De) % E);
-  for (int i = tid; i < T * Th; i += MMOE_THREADS) bt[i] = __ldg(P.bt[i / Th] + i % Th);
-  for (int k = tid; k < T; k += MMOE_THREADS) bo[k] = __ldg(P.bo[k]);
-  __syncthreads();   // mbarrier initialised before anyone waits on it
-  ptx::mbar_wait(&bar, 0);
-  // ---- 1: fused expert + gate GEMM; a warp computes 4 (row, batch) outputs at once (lanes split D,
-  // four independent accumulators and shuffle trees in flight: the chain latency is paid once per 4)
-  constexpr int kO = 4, kWarps = MMOE_THREADS / 32;
-  for (int o0 = warp * kO; o0 < R * B; o0 += kWarps * kO) {
-    float s[kO] = {0.f, 0.f, 0.f, 0.f};
-    for (int k = lane; k < D; k += 32) {
+  long long tk[7];
+  const bool dbg = P.pad != 0;   // debug timeline (SOUFFLE_MMOE_DEBUG): thread 0 prints phase times
+  if (dbg && tid == 0) tk[0] = clock64();
+  // ---- every parameter into shared memory with plain 16-byte loads by all 1024 threads (~59 KB: 4
+  // loads per thread, all in flight -- one L2 round trip; 14 serial bulk-copy issues by one thread
+  // measured ~7 us).  Parameter-array indices are compile-time (unrolled, predicated) everywhere: a
+  // runtime index into the __grid_constant__ block would copy it to local memory
+  auto copy16 = [&](char* dst, const void* src, int bytes) {
+    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    uint4* d4 = reinterpret_cast<uint4*>(dst);
+    for (int v = tid; v < (bytes >> 4); v += MMOE_THREADS) d4[v] = __ldg(s4 + v);
+  };
 #pragma unroll
-      for (int j = 0; j < kO; ++j) {
-        const int o = o0 + j;
-        if (o < R * B) s[j] = fmaf(xs[(o / R) * D + k], wsm(W1, (int64_t)(o % R) * D + k, f32), s[j]);
-      }
+  for (int e = 0; e < MMOE_MAX_E; ++e)
+    if (e < E) copy16(W1 + (int64_t)e * De * D * es, P.We[e], De * D * es);
+#pragma unroll
+  for (int k = 0; k < MMOE_MAX_T; ++k)
+    if (k < T) {
+      copy16(W1 + (int64_t)(E * De + k * E) * D * es, P.Wg[k], E * D * es);
+      copy16(Wt + (int64_t)k * Th * De * es, P.Wt[k], Th * De * es);
+      copy16(Wo + (int64_t)k * Th * es, P.Wo[k], Th * es);
     }
+  for (int i = tid; i < B * D; i += MMOE_THREADS) xs[i] = __ldg(P.x + i);
 #pragma unroll
-    for (int off = 16; off > 0; off >>= 1)
+  for (int e = 0; e < MMOE_MAX_E; ++e)
+    if (e < E)
+      for (int j = tid; j < De; j += MMOE_THREADS) b1[e * De + j] = __ldg(P.be[e] + j);
 #pragma unroll
-      for (int j = 0; j < kO; ++j) s[j] += __shfl_xor_sync(0xffffffffu, s[j], off);
-    if (lane < kO && o0 + lane < R * B) {
-      const int o = o0 + lane, r = o % R, b = o / R;
-      const float sl = lane == 0 ? s[0] : lane == 1 ? s[1] : lane == 2 ? s[2] : s[3];
-      const float v = sl + b1[r];
+  for (int k = 0; k < MMOE_MAX_T; ++k)
+    if (k < T) {
+      for (int j = tid; j < E; j += MMOE_THREADS) b1[E * De + k * E + j] = __ldg(P.bg[k] + j);
+      for (int j = tid; j < Th; j += MMOE_THREADS) bt[k * Th + j] = __ldg(P.bt[k] + j);
+      if (tid == 0) bo[k] = __ldg(P.bo[k]);
+    }
+  __syncthreads();
+  if (dbg && tid == 0) tk[1] = clock64();
+  if (dbg && tid == 0) tk[2] = clock64();
+  // ---- 1: fused expert + gate GEMM, 4 threads per (row, batch) output, k interleaved by 4 (the 8
+  // outputs of a warp hit 32 distinct banks: row stride D = 100 floats = 4 banks), 2 shuffles
+  for (int base = warp * 32; base < 4 * R * B; base += MMOE_THREADS) {   // warp-uniform trip count
+    const int it = base + lane, o = it >> 2, part = it & 3;
+    const bool valid = o < R * B;
+    const int r = valid ? o % R : 0, b = valid ? o / R : 0;
+    const float* xr = xs + b * D;
+    float s = 0.f;
+    if (valid)
+      for (int k = part; k < D; k += 4) s = fmaf(xr[k], wsm(W1, r * D + k, f32), s);
+    s += __shfl_xor_sync(0xffffffffu, s, 1);
+    s += __shfl_xor_sync(0xffffffffu, s, 2);
+    if (valid && part == 0) {
+      const float v = s + b1[r];
       o1[b * R + r] = r < E * De ? fmaxf(v, 0.f) : v;
     }
   }
   __syncthreads();
-  // ---- 2: per-task softmax over the experts (in place, max-subtracted)
-  if (tid < B * T) {
-    const int b = tid / T, k = tid % T;
+  if (dbg && tid == 0) tk[3] = clock64();
+  // ---- 2: per-task softmax over the experts (in place, max-subtracted): warp (b, k), lane = expert
+  if (warp < B * T) {
+    const int b = warp / T, k = warp % T;
     float* g = o1 + b * R + E * De + k * E;
-    float m = -INFINITY;
-    for (int e = 0; e < E; ++e) m = fmaxf(m, g[e]);
-    float z = 0.f;
-    for (int e = 0; e < E; ++e) {
-      g[e] = expf(g[e] - m);
-      z += g[e];
-    }
-    for (int e = 0; e < E; ++e) g[e] = g[e] / z;
+    const float v = lane < E ? g[lane] : -INFINITY;
+    float m = v;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, off));
+    const float ex = lane < E ? expf(v - m) : 0.f;
+    float z = ex;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) z += __shfl_xor_sync(0xffffffffu, z, off);
+    if (lane < E) g[lane] = ex / z;
   }
   __syncthreads();
   // ---- 3: mixtures f_k = sum_e g_k[e] * E_e (the graph's add chain, in expert order)
@@ -119,19 +132,34 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
     f[i] = acc;
   }
   __syncthreads();
-  // ---- 4: towers
-  for (int i = tid; i < B * T * Th; i += MMOE_THREADS) {
+  if (dbg && tid == 0) tk[4] = clock64();
+  // ---- 4: towers: 8 lanes per hidden unit (products split over De, shuffle sum)
+  for (int base = warp * 32; base < B * T * Th * 8; base += MMOE_THREADS) {   // warp-uniform trip count
+    const int i0 = base + lane, i = i0 >> 3, part = i0 & 7;
+    const bool valid = i0 < B * T * Th * 8;
     const int b = i / (T * Th), k = (i / Th) % T, r = i % Th;
     float s = 0.f;
-    for (int j = 0; j < De; ++j) s = fmaf(f[(b * T + k) * De + j], wsm(Wt, (int64_t)(k * Th + r) * De + j, f32), s);
-    h1[i] = fmaxf(s + bt[k * Th + r], 0.f);
+    if (valid)
+      for (int j = part; j < De; j += 8) s = fmaf(f[(b * T + k) * De + j], wsm(Wt, (k * Th + r) * De + j, f32), s);
+    s += __shfl_xor_sync(0xffffffffu, s, 4);
+    s += __shfl_xor_sync(0xffffffffu, s, 2);
+    s += __shfl_xor_sync(0xffffffffu, s, 1);
+    if (valid && part == 0) h1[i] = fmaxf(s + bt[k * Th + r], 0.f);
   }
   __syncthreads();
-  if (tid < B * T) {
-    const int b = tid / T, k = tid % T;
-    float s = 0.f;
-    for (int r = 0; r < Th; ++r) s = fmaf(h1[(b * T + k) * Th + r], wsm(Wo, k * Th + r, f32), s);
-    P.y[k][b] = s + bo[k];
+  if (warp < B * T) {
+    const int b = warp / T, k = warp % T;
+    float s = lane < Th ? h1[(b * T + k) * Th + lane] * wsm(Wo, k * Th + lane, f32) : 0.f;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+#pragma unroll
+    for (int kk = 0; kk < MMOE_MAX_T; ++kk)
+      if (kk == k && lane == 0) P.y[kk][b] = s + bo[k];
+  }
+  if (dbg && tid == 0) {
+    tk[5] = clock64();
+    printf("mmoe clocks: params+issue %lld | bulk wait %lld | gemm %lld | softmax+mix %lld | towers %lld\n",
+           tk[1] - tk[0], tk[2] - tk[1], tk[3] - tk[2], tk[4] - tk[3], tk[5] - tk[4]);
   }
 }
 

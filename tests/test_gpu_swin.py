@@ -86,23 +86,27 @@ def _swin_b_child(batch):
           float(np.sqrt(np.mean(ref ** 2))), "pattern swin: batch" in plan.describe())
 
 
-@pytest.mark.parametrize("batch", [1, 8])
-def test_swin_b_full_size(batch, record_err):
+@pytest.mark.parametrize("batch,two_sm", [(1, False), (8, False), (8, True)])
+def test_swin_b_full_size(batch, two_sm, record_err):
     """Full Swin-B (BASELINE.json configs[4]) at batch 1 and 8 through the pattern kernels against the
-    bf16-operand oracle, in a fresh process (isolated from the kernels the other tests ran)."""
+    bf16-operand oracle, in a fresh process (isolated from the kernels the other tests ran); batch 8
+    also with the opt-in 2-SM (cta_group::2) GEMM tiles, which its stage-1/2 GEMMs select."""
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     code = "import sys; sys.path.insert(0, %r); sys.path.insert(0, %r); import test_gpu_swin as t; t._swin_b_child(%d)" % (
         root, os.path.join(root, "tests"), batch)
-    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=900, cwd=root)
+    env = dict(os.environ)
+    if two_sm:
+        env["SOUFFLE_SWIN_2SM"] = "1"
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=900, cwd=root, env=env)
     line = [ln for ln in r.stdout.splitlines() if ln.startswith("RESULT")]
     assert line, r.stderr[-2000:]
     _, b, n, e1, e2, rms, pat = line[0].split()
     assert (int(b), int(n)) == (batch, 1000) and pat == "True"
     assert float(e2) <= 2e-2
-    record_err(float(e1), 2e-2, batch=batch, rms=float(rms))
+    record_err(float(e1), 2e-2, batch=batch, rms=float(rms), two_sm=two_sm)
 
 
 def _swin_b64_child():
