@@ -124,6 +124,13 @@ void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
   if (g.outputs != mp.y) return no("outputs are not the task towers");
   if (mp.E > MMOE_MAX_E || mp.T > MMOE_MAX_T || mp.B > MMOE_MAX_B) return no("too many experts / tasks / rows");
   if (mp.B * mp.T > MMOE_THREADS / 32 || mp.Th > 32) return no("batch x tasks > warps or tower width > 32");
+  if (1 + mp.E + 3 * mp.T > 32) return no("more than 32 parameter segments (one warp builds the staging table)");
+  {   // parameter staging (kernels/mmoe.cu): <= 4 x 1024 16-byte weight units, <= 1024 vector elements
+    const int64_t es2 = mp.w_f32 ? 4 : 2;
+    const int64_t w16 = ((int64_t)mp.E * mp.De * mp.D + (int64_t)mp.T * (mp.E * mp.D + mp.Th * mp.De + mp.Th)) * es2 / 16;
+    const int64_t vec = (int64_t)mp.B * mp.D + (int64_t)mp.E * mp.De + (int64_t)mp.T * (mp.E + mp.Th + 1);
+    if (w16 > 4 * MMOE_THREADS || vec > MMOE_THREADS) return no("parameters exceed the staging capacity");
+  }
   const int epv = mp.w_f32 ? 4 : 8;   // weight tensors are staged by bulk copies of 16-byte multiples
   if ((int64_t)mp.De * mp.D % epv || (int64_t)mp.E * mp.D % epv || (int64_t)mp.Th * mp.De % epv || mp.Th % epv)
     return no("weight tensor sizes must be multiples of 16 bytes");

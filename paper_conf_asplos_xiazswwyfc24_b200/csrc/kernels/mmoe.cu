@@ -55,37 +55,94 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   long long tk[7];
   const bool dbg = P.pad != 0;   // debug timeline (SOUFFLE_MMOE_DEBUG): thread 0 prints phase times
   if (dbg && tid == 0) tk[0] = clock64();
-  // ---- every parameter into shared memory with plain 16-byte loads by all 1024 threads (~59 KB: 4
-  // loads per thread, all in flight -- one L2 round trip; 14 serial bulk-copy issues by one thread
-  // measured ~7 us).  Parameter-array indices are compile-time (unrolled, predicated) everywhere: a
-  // runtime index into the __grid_constant__ block would copy it to local memory
-  auto copy16 = [&](char* dst, const void* src, int bytes) {
-    const uint4* s4 = reinterpret_cast<const uint4*>(src);
-    uint4* d4 = reinterpret_cast<uint4*>(dst);
-    for (int v = tid; v < (bytes >> 4); v += MMOE_THREADS) d4[v] = __ldg(s4 + v);
-  };
+  // ---- every parameter into shared memory with plain loads by all 1024 threads, all in flight at
+  // once (one L2 round trip).  Thread 0 first writes a segment table (source, destination, length)
+  // -- 16-byte weight segments and 4-byte vector segments -- then every thread loads its (up to 4 +
+  // 1) elements of the concatenation before storing any (14 serial bulk-copy issues measured ~7 us,
+  // per-segment load/store loops ~11 us).
+  constexpr int kSeg = MMOE_MAX_E + 3 * MMOE_MAX_T + 1;
+  __shared__ const char* s_src[2][kSeg];
+  __shared__ char* s_dst[2][kSeg];
+  __shared__ int s_pre[2][kSeg + 1];
+  __shared__ int s_nseg[2];
+  if (warp == 0) {
+    // segment table, one segment per lane (weights: We[0..E) then per task Wg, Wt, Wo; vectors: x,
+    // be[0..E) then per task bg, bt, bo), lengths prefix-summed with a warp scan
+    const int nw = E + 3 * T, nv = 1 + E + 3 * T;
+    for (int t = 0; t < 2; ++t) {
+      const int n = t == 0 ? nw : nv;
+      const char* src = nullptr;
+      char* dst = nullptr;
+      int units = 0;
+      if (lane < n) {
+        if (t == 0) {
+          if (lane < E) {
+            src = (const char*)P.We[lane]; dst = W1 + (int64_t)lane * De * D * es; units = De * D * es / 16;
+          } else {
+            const int k = (lane - E) / 3, which = (lane - E) % 3;
+            if (which == 0) { src = (const char*)P.Wg[k]; dst = W1 + (int64_t)(E * De + k * E) * D * es; units = E * D * es / 16; }
+            else if (which == 1) { src = (const char*)P.Wt[k]; dst = Wt + (int64_t)k * Th * De * es; units = Th * De * es / 16; }
+            else { src = (const char*)P.Wo[k]; dst = Wo + (int64_t)k * Th * es; units = Th * es / 16; }
+          }
+        } else {
+          if (lane == 0) { src = (const char*)P.x; dst = (char*)xs; units = B * D; }
+          else if (lane <= E) { src = (const char*)P.be[lane - 1]; dst = (char*)(b1 + (lane - 1) * De); units = De; }
+          else {
+            const int k = (lane - 1 - E) / 3, which = (lane - 1 - E) % 3;
+            if (which == 0) { src = (const char*)P.bg[k]; dst = (char*)(b1 + E * De + k * E); units = E; }
+            else if (which == 1) { src = (const char*)P.bt[k]; dst = (char*)(bt + k * Th); units = Th; }
+            else { src = (const char*)P.bo[k]; dst = (char*)(bo + k); units = 1; }
+          }
+        }
+      }
+      int incl = units;   // inclusive scan over the lanes
 #pragma unroll
-  for (int e = 0; e < MMOE_MAX_E; ++e)
-    if (e < E) copy16(W1 + (int64_t)e * De * D * es, P.We[e], De * D * es);
-#pragma unroll
-  for (int k = 0; k < MMOE_MAX_T; ++k)
-    if (k < T) {
-      copy16(W1 + (int64_t)(E * De + k * E) * D * es, P.Wg[k], E * D * es);
-      copy16(Wt + (int64_t)k * Th * De * es, P.Wt[k], Th * De * es);
-      copy16(Wo + (int64_t)k * Th * es, P.Wo[k], Th * es);
+      for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += y;
+      }
+      if (lane < n) {
+        s_src[t][lane] = src;
+        s_dst[t][lane] = dst;
+        s_pre[t][lane] = incl - units;
+      }
+      if (lane == n - 1) {
+        s_pre[t][n] = incl;
+        s_nseg[t] = n;
+      }
     }
-  for (int i = tid; i < B * D; i += MMOE_THREADS) xs[i] = __ldg(P.x + i);
+  }
+  __syncthreads();
+  {
+    constexpr int kW = 4;   // 16-byte units per thread (the MMoE parameters are <= 4 x 1024 x 16 B)
+    uint4 wv[kW];
+    int ws[kW], wo[kW];
+    float fv;
+    int fs = -1, fo = 0;
 #pragma unroll
-  for (int e = 0; e < MMOE_MAX_E; ++e)
-    if (e < E)
-      for (int j = tid; j < De; j += MMOE_THREADS) b1[e * De + j] = __ldg(P.be[e] + j);
-#pragma unroll
-  for (int k = 0; k < MMOE_MAX_T; ++k)
-    if (k < T) {
-      for (int j = tid; j < E; j += MMOE_THREADS) b1[E * De + k * E + j] = __ldg(P.bg[k] + j);
-      for (int j = tid; j < Th; j += MMOE_THREADS) bt[k * Th + j] = __ldg(P.bt[k] + j);
-      if (tid == 0) bo[k] = __ldg(P.bo[k]);
+    for (int j = 0; j < kW; ++j) {
+      const int idx = tid + j * MMOE_THREADS;
+      ws[j] = -1;
+      if (idx < s_pre[0][s_nseg[0]]) {
+        int sg = 0;
+        while (s_pre[0][sg + 1] <= idx) ++sg;
+        ws[j] = sg;
+        wo[j] = idx - s_pre[0][sg];
+        wv[j] = __ldg(reinterpret_cast<const uint4*>(s_src[0][sg]) + wo[j]);
+      }
     }
+    if (tid < s_pre[1][s_nseg[1]]) {   // vectors: at most one fp32 per thread
+      int sg = 0;
+      while (s_pre[1][sg + 1] <= tid) ++sg;
+      fs = sg;
+      fo = tid - s_pre[1][sg];
+      fv = __ldg(reinterpret_cast<const float*>(s_src[1][sg]) + fo);
+    }
+#pragma unroll
+    for (int j = 0; j < kW; ++j)
+      if (ws[j] >= 0) reinterpret_cast<uint4*>(s_dst[0][ws[j]])[wo[j]] = wv[j];
+    if (fs >= 0) reinterpret_cast<float*>(s_dst[1][fs])[fo] = fv;
+  }
   __syncthreads();
   if (dbg && tid == 0) tk[1] = clock64();
   if (dbg && tid == 0) tk[2] = clock64();
