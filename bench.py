@@ -177,8 +177,9 @@ def build_bert(device_index, flags=0):
     x = synth.bert_input(cfg)
     w = synth.bert_weights(cfg)
     g, X, plist, y = M.bert(cfg)
+    dev = L.device_query(device_index)
     t0 = time.perf_counter()
-    plan = g.partition(L.device_query(device_index), flags)
+    plan = g.partition(dev, flags)
     build_bert.plan_s = time.perf_counter() - t0   # analysis + partition + lowering (host)
     feed = {X: x}
     for names, wl in zip(plist, w):

@@ -410,3 +410,25 @@ def swin(cfg):
     names["Wh"], names["bh"] = Wh, bh
     b.out(y)
     return b.spec(), names, x, y
+
+
+def se_module(cfg):
+    """EfficientNet squeeze-and-excitation sub-module (Fig. 5; torchvision
+    SqueezeExcitation with SiLU / Sigmoid): y = x * sigmoid(fc2(silu(fc1(mean_rows(x))))).
+    x [H*W, C] (NHWC, batch 1).  Returns (spec, names, x id, y id)."""
+    HW, C, S = cfg["hw"] * cfg["hw"], cfg["channels"], cfg["squeeze"]
+    b = SpecBuilder()
+    x = b.ph((HW, C), const=0)
+    p = b.red("mean", x, 0)                    # [1, C] global average pool
+    W1 = b.ph((S, C))
+    h = b.mm(p, W1, 1, "f32")
+    b1 = b.ph((S,))
+    h = b.ew("add", h, b1)
+    h = b.ew("mul", h, b.ew("sigmoid", h))     # SiLU
+    W2 = b.ph((C, S))
+    g = b.mm(h, W2, 1, "f32")
+    b2 = b.ph((C,))
+    g = b.ew("sigmoid", b.ew("add", g, b2))
+    y = b.ew("mul", x, g)                      # channel-wise rescale (broadcast over rows)
+    b.out(y)
+    return b.spec(), dict(x=x, W1=W1, b1=b1, W2=W2, b2=b2), x, y

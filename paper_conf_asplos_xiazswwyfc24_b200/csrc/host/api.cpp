@@ -484,6 +484,12 @@ souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t
       if (barriers) *barriers = P.bert.nstages - 1;
       return;
     }
+    if (P.se.on) {
+      if (launches) *launches = 1;
+      if (stages) *stages = 4;
+      if (barriers) *barriers = 3;
+      return;
+    }
     if (P.swin.on) {   // one kernel per fused subprogram, replayed as one CUDA graph
       if (launches) *launches = P.swin.launches;
       if (stages) *stages = P.swin.launches;

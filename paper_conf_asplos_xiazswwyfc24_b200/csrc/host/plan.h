@@ -9,6 +9,7 @@
 #include "lstm.h"
 #include "mmoe.h"
 #include "swin.h"
+#include "se.h"
 #include "ir.h"
 
 namespace souffle {
@@ -62,6 +63,7 @@ struct Plan {
   LstmPlan lstm;                    // pattern lowering (lstm.on: kernels/lstm.cu runs the program)
   MmoePlan mmoe;                    // pattern lowering (mmoe.on: kernels/mmoe.cu runs the program)
   SwinPlan swin;                    // pattern lowering (swin.on: kernels/swin.cu, one CUDA graph)
+  SePlan se;                        // pattern lowering (se.on: kernels/se.cu, EfficientNet M0-M9)
   ~Plan();
 };
 

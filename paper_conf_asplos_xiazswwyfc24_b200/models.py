@@ -320,3 +320,24 @@ def swin(cfg):
     names["Wh"], names["bh"] = Wh, bh
     g.mark_output(y)
     return g, names, x, y
+
+
+# ---------------------------------------------------------------- EfficientNet SE sub-module (Fig. 5)
+def se_module(cfg):
+    """y = x * sigmoid(fc2(silu(fc1(mean_rows(x))))), x [H*W, C] (same node order as oracle.graphs)."""
+    HW, C, S = cfg["hw"] * cfg["hw"], cfg["channels"], cfg["squeeze"]
+    g = L.Graph()
+    x = g.placeholder((HW, C), L.F32, const=False)
+    p = g.reduce("mean", x, 0, True)
+    W1 = g.placeholder((S, C))
+    h = g.matmul(p, W1, True, L.F32)
+    b1 = g.placeholder((S,))
+    h = g.ew("add", h, b1)
+    h = g.ew("mul", h, g.ew("sigmoid", h))
+    W2 = g.placeholder((C, S))
+    gt = g.matmul(h, W2, True, L.F32)
+    b2 = g.placeholder((C,))
+    gt = g.ew("sigmoid", g.ew("add", gt, b2))
+    y = g.ew("mul", x, gt)
+    g.mark_output(y)
+    return g, dict(x=x, W1=W1, b1=b1, W2=W2, b2=b2), x, y

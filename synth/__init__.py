@@ -227,3 +227,27 @@ def spec_inputs(spec: dict, seed: int, integer: bool = False) -> dict:
         else:
             out[i] = normal(seed * 7919 + i, tuple(n["shape"]), std=0.5, dtype=n["dtype"])
     return out
+
+
+# ---------------------------------------------------------------- EfficientNet sub-modules M0-M9
+# PAPER.md Fig. 5 / Fig. 6 (L1511-1564): the squeeze-and-excitation sub-module of EfficientNet-b0's
+# MBConv blocks "repeats many times with different input sizes (M0 to M9)".  The 10 distinct
+# (expanded channels C, feature map H x H, squeeze channels S) of efficientnet_b0's 16 blocks
+# (torchvision: S = max(1, block input channels // 4)), in network order (reading R20).
+SE_CONFIGS = [
+    dict(name=f"M{i}", hw=h, channels=c, squeeze=s)
+    for i, (c, h, s) in enumerate([(32, 112, 8), (96, 56, 4), (144, 56, 6), (144, 28, 6), (240, 28, 10),
+                                   (240, 14, 10), (480, 14, 20), (672, 14, 28), (672, 7, 28), (1152, 7, 48)])
+]
+
+
+def se_input(cfg: dict, seed: int = INPUT_SEED) -> np.ndarray:
+    """x [H*W, C] fp32 ~ N(0, 1): the depthwise-conv output the sub-module rescales (NHWC, batch 1)."""
+    return normal(seed, (cfg["hw"] * cfg["hw"], cfg["channels"]))
+
+
+def se_params(cfg: dict) -> dict:
+    """fc1 [S, C] ~ N(0, 1/C), b1 N(0, 0.02^2); fc2 [C, S] ~ N(0, 1/S), b2 N(0, 0.02^2); fp32."""
+    C, S = cfg["channels"], cfg["squeeze"]
+    return dict(W1=normal(701, (S, C), std=1.0 / np.sqrt(C)), b1=normal(702, (S,), std=0.02),
+                W2=normal(703, (C, S), std=1.0 / np.sqrt(S)), b2=normal(704, (C,), std=0.02))
