@@ -30,7 +30,8 @@ enum {
   BERT_COMPUTE = 256,
   BW_SLOTS = 5,                // weight ring: 5 x 16 KB; a slot holds 16 KB / (n_tile * 128 B) K-chunks
   BW_SLOT_BYTES = 16384,
-  BA_SLOTS = 8,                // A operand ring: 8 x (128 rows x 64 K bf16); also the epilogue staging tile
+  BA_SLOTS = 7,                // A operand ring: 7 x (128 rows x 64 K bf16) >= the 6 K chunks a
+                               // cluster-pair task streams; also the attention operands and staging
   BA_SLOT_BYTES = 16384,
   B_CTRL_BYTES = 2048,         // control block + two staged stage descriptors
   B_AREGION = BA_SLOTS * BA_SLOT_BYTES,   // also holds the attention operands Q, K, V^T, P (80 KB)

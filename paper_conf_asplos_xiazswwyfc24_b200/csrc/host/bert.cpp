@@ -26,6 +26,7 @@ extern thread_local std::string g_err;
 souffle_status fail(souffle_status c, const std::string& m);
 cudaError_t bert_launch(const BertParams& prm, int grid, bool pairs, cudaStream_t s);
 cudaError_t bert_max_active(int* blocks);
+cudaError_t bert_max_clusters(int grid, int* clusters);
 
 namespace {
 
@@ -552,6 +553,18 @@ souffle_status bert_run(Plan& p, void* ws, void* stream) {
   need = std::max(need, bp.heads);
   if (max_active < 1 || grid < need)
     return fail(SOUFFLE_E_RESOURCE, "BERT persistent kernel needs " + std::to_string(need) + " co-resident CTAs");
+  if (bp.pairs) {   // every CTA pair must be co-resident (the launch is not cooperative, see bert_launch)
+    static int max_clusters = -1;
+    if (max_clusters < 0) {
+      int c = 0;
+      cudaError_t e = bert_max_clusters(grid, &c);
+      if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("cluster occupancy query: ") + cudaGetErrorString(e));
+      max_clusters = c;
+    }
+    if (max_clusters * 2 < grid)
+      return fail(SOUFFLE_E_RESOURCE, "only " + std::to_string(max_clusters) + " CTA pairs can be co-resident, need " +
+                                          std::to_string(grid / 2));
+  }
   char* base = (char*)ws;
   BertParams prm;
   std::memset(&prm, 0, sizeof(prm));

@@ -875,16 +875,41 @@ cudaError_t bert_launch(const BertParams& prm, int grid, bool pairs, cudaStream_
   cfg.blockDim = dim3(BERT_THREADS);
   cfg.dynamicSmemBytes = B_SMEM;
   cfg.stream = s;
-  cudaLaunchAttribute at[2];
-  at[0].id = cudaLaunchAttributeCooperative;
-  at[0].val.cooperative = 1;
-  at[1].id = cudaLaunchAttributeClusterDimension;   // CTA pairs (cluster-pair split-K stages)
-  at[1].val.clusterDim.x = 2;
-  at[1].val.clusterDim.y = 1;
-  at[1].val.clusterDim.z = 1;
+  // Without clusters the launch is cooperative (the runtime checks co-residency).  With CTA pairs it
+  // is a plain cluster launch whose co-residency bert_max_clusters() checked at plan time (a
+  // cooperative cluster launch is refused under the profiler)
+  cudaLaunchAttribute at[1];
+  if (pairs) {
+    at[0].id = cudaLaunchAttributeClusterDimension;   // CTA pairs (cluster-pair split-K stages)
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+  } else {
+    at[0].id = cudaLaunchAttributeCooperative;
+    at[0].val.cooperative = 1;
+  }
   cfg.attrs = at;
-  cfg.numAttrs = pairs ? 2 : 1;
+  cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, bert::bert_kernel, prm);
+}
+
+// how many CTA-pair clusters of the BERT kernel can be resident at once (all must be: spin barriers)
+cudaError_t bert_max_clusters(int grid, int* clusters) {
+  cudaError_t e = cudaFuncSetAttribute(bert::bert_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, B_SMEM);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(bert::bert_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 0);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(BERT_THREADS);
+  cfg.dynamicSmemBytes = B_SMEM;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 2;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaOccupancyMaxActiveClusters(clusters, bert::bert_kernel, &cfg);
 }
 
 cudaError_t bert_max_active(int* blocks) {

@@ -82,12 +82,8 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
   float h = 0.f;
   __syncthreads();
 
-  auto stamp = [&](int t, int k) {
-    if (P.prof && blockIdx.x == P.prof_cta && tid == 0) {
-      unsigned long long g;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
-      P.prof[4 * t + k] = g;
-    }
+  auto stamp = [&](int t, int k) {   // debug timeline: SM clock cycles (%globaltimer ticks in 256 ns steps)
+    if (P.prof && blockIdx.x == P.prof_cta && tid == 0) P.prof[4 * t + k] = (unsigned long long)clock64();
   };
   const unsigned gen = *(volatile unsigned*)P.gen;   // written by the previous launch's last CTA
   const unsigned tag0 = gen * (unsigned)(T + 1) + 1u;
@@ -186,6 +182,7 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
       uint2* dst = P.hbuf + ((int64_t)l * T + t) * H + unit;
       asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(dst), "l"(w64) : "memory");
     }
+    stamp(t, 3);
   }
   if (warp == 0 && own) {
     Ly.h_n[unit] = h;

@@ -34,11 +34,11 @@ T = cfg["steps"]
 buf = (C.c_uint64 * (4 * T))()
 got = C.c_int32()
 L.check(plan.lib.souffle_plan_read_profile_raw(plan.h, C.c_void_p(s.ws.data_ptr()), buf, 4 * T, C.byref(got)))
-st = np.array(list(buf), dtype=np.float64).reshape(T, 4)
+st = np.array(list(buf), dtype=np.float64).reshape(T, 4) / 1.965   # SM cycles -> ns (1965 MHz under load)
 t0 = st[0, 0]
 for t in list(range(0, 6)) + list(range(T - 3, T)):
     print(f"t={t:3d} start {(st[t,0]-t0)/1e3:8.2f} operands +{(st[t,1]-st[t,0])/1e3:5.2f} gemv +{(st[t,2]-st[t,1])/1e3:5.2f}"
-          f" next-start +{((st[t+1,0]-st[t,2])/1e3 if t + 1 < T else 0):5.2f}")
+          f" cell+publish +{(st[t,3]-st[t,2])/1e3:5.2f} next-start +{((st[t+1,0]-st[t,3])/1e3 if t + 1 < T else 0):5.2f}")
 d = np.diff(st[:, 0]) / 1e3
 print("mean step", d.mean(), "operands wait mean", ((st[:, 1] - st[:, 0]) / 1e3).mean(), "gemv mean",
-      ((st[:, 2] - st[:, 1]) / 1e3).mean())
+      ((st[:, 2] - st[:, 1]) / 1e3).mean(), "cell+publish mean", ((st[:, 3] - st[:, 2]) / 1e3).mean())

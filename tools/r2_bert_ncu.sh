@@ -1,0 +1,12 @@
+#!/bin/bash
+mkdir -p gpurun_out
+python -c "from paper_conf_asplos_xiazswwyfc24_b200.build import build; build()" > gpurun_out/build.log 2>&1
+timeout 600 python -m pytest tests/test_gpu_bert_stages.py tests/test_gpu_parity.py -q -x -m gpu -k "bert or stage or layernorm or bias" > gpurun_out/pytest_bert.txt 2>&1
+echo "rc=$?" >> gpurun_out/pytest_bert.txt
+timeout 300 python tools/sweep_bert.py "" > gpurun_out/sweep_now.txt 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/r02_launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-v0 --no-models > gpurun_out/r02_ncu_launch.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:bert_kernel -s 1 -c 1 -o gpurun_out/r02_prof_bert python tools/run_once.py bert_base 0 0 2 > gpurun_out/r02_ncu_full.log 2>&1
+timeout 1200 python tools/ablation_se.py gpurun_out/se_ablation.jsonl > gpurun_out/se_ablation.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_se.py -q -m gpu > gpurun_out/pytest_se.txt 2>&1
+echo "rc=$?" >> gpurun_out/pytest_se.txt
+echo done
