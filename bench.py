@@ -458,6 +458,29 @@ def main():
                          "empty_kernel_graph_replay_us": graph_us(lambda: dummy.add_(1)),
                          "paper_a100_us": 14.0}
         del msess, mplan
+        # EfficientNet squeeze-excitation sub-modules M0-M9 (Fig. 5/6): the
+        # pattern kernel (global sync + data reuse) against the unfused one-kernel-per-TE path
+        progress("EfficientNet SE sub-modules")
+        from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+        from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+        from paper_conf_asplos_xiazswwyfc24_b200.session import session as _session
+        import synth as _synth
+        se_rows = []
+        for cfg in _synth.SE_CONFIGS:
+            xs_, ps_ = _synth.se_input(cfg), _synth.se_params(cfg)
+            g_, nm_, gx_, gy_ = M.se_module(cfg)
+            row = {"module": cfg["name"], "hw": cfg["hw"], "c": cfg["channels"]}
+            for key, fl in (("data_reuse_us", 0), ("unfused_us", L.FLAG_UNFUSED)):
+                pl_ = g_.partition(L.device_query(local), fl)
+                ss_ = _session(g_, pl_, {nm_[k]: ps_[k] for k in ps_} | {gx_: xs_}, [gy_], device=f"cuda:{local}")
+                row[key] = statistics.median(time_steps(ss_, 20, 3, flush, stream)) * 1e3
+                del ss_, pl_
+            row["speedup"] = row["unfused_us"] / row["data_reuse_us"]
+            se_rows.append(row)
+        extra["efficientnet_se"] = {"workload": "EfficientNet-b0 squeeze-excitation sub-modules M0-M9 (fp32, batch 1)",
+                                    "modules": se_rows,
+                                    "geomean_speedup_vs_unfused": float(np.exp(np.mean([np.log(r["speedup"]) for r in se_rows]))),
+                                    "paper_a100": "Fig. 6: 1.31x global sync, 1.84x data reuse over unfused (avg)"}
         # Swin-B runs in a child process (fresh CUDA context) with a time limit: a launch that trips a
         # kernel watchdog must not take the whole bench line with it
         progress("Swin-B (child process)")
