@@ -38,6 +38,15 @@ enum Fn : int16_t {
 
 enum { NREG = 4, CHUNK = 8, MAX_RED = 4, MAX_BUFS = 480, EXEC_THREADS = 256, EXEC_SMEM = 136 * 1024 };
 
+// Software-managed shared-memory tensor cache (§6.5, "tensor reuse
+// optimization"): fp32 words above the EXEC_SMEM working area, so GEMM / attention stages between a
+// tensor's producer and its consumers leave it intact.  At most EXEC_CACHE_FLOATS (88 KB: a CTA stays
+// within the 227 KB opt-in limit); by default EXEC_CACHE_DEFAULT_FLOATS (24 KB), which still fits the
+// 164 KB shared-memory carveout the working area needs -- a larger cache shrinks L1, which the
+// interpreter's index-table and weight loads use (measured on Swin-B / BERT V3).
+enum { EXEC_CACHE_FLOATS = 22528, EXEC_CACHE_DEFAULT_FLOATS = 6144 };
+enum CacheMode : int16_t { CM_FILL = 1, CM_NOSTORE = 2 };
+
 // Address of a tensor element at domain point (r, c):
 //   element offset = base + row(r) + col(c)
 //   mode 0 affine:    row(r) = r*rs,            col(c) = c*cs
@@ -54,6 +63,14 @@ struct Addr {
   int32_t rtab, ctab, ftab, ncols;
   int16_t cg;     // 1: tensor is written inside the run -> coherent (L2) loads
   int16_t cvec;   // mode 1: col(c0 + j) == col(c0) + j within every aligned chunk of CHUNK columns
+  // tensor cache (row-block stages, mode 0 only): cache = float offset of the tensor's slot in the
+  // cache region + 1 (0: not cached).  Domain row r belongs to row block r / crb, which CTA
+  // (r / crb) % gridDim.x owns in every row-block stage of the launch; element (r, c) lives at
+  // slot + ((r / crb) / gridDim.x) * crb * rs + (r % crb) * rs + c * cs.  A load reads the slot
+  // (cmode & CM_FILL: reads global memory and deposits the chunk); a store writes the slot, rounded
+  // to dtype, and global memory unless cmode & CM_NOSTORE (every consumer hits).
+  int32_t cache;
+  int16_t crb, cmode;
 };
 
 struct Ins {
@@ -111,6 +128,12 @@ struct Stage {
   float at_scale;
   int32_t barrier_after;            // the next stage of the same launch starts with a grid barrier
   int32_t at_add[2];                // ATTN: Addr of additive score terms at (b*S + i, j), -1 if none
+  // REDUCE / EW: rows per row block.  CTA b owns row blocks b, b + grid, ... (REDUCE: always, a warp
+  // per 32/G rows; EW: when rblk > 0, else chunk t goes to thread t mod (grid * threads)).  Stages
+  // of one launch with equal rows and rblk hand rows to the same CTA: a dependency between them is
+  // CTA-local (no grid barrier, tensor cache hits).
+  int32_t rblk;
+  int32_t pad_rb[3];
 };
 
 struct Launch {

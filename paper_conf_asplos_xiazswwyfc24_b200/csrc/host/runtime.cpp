@@ -239,6 +239,9 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
       if (cap < 1) return fail(SOUFFLE_E_RESOURCE, "persistent kernel cannot be resident");
       if (grid > cap) grid = cap;  // persistent stages loop over their tasks
     }
+    // the tensor cache's slot placement assumes the planned grid (one CTA per SM)
+    if (L.smem > EXEC_SMEM && grid != L.grid)
+      return fail(SOUFFLE_E_RESOURCE, "tensor-cache launch needs its planned grid (plan made for another device?)");
     prm.first = L.first;
     prm.count = L.count;
     prm.cooperative = L.cooperative;

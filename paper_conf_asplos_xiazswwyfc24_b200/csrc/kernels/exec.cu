@@ -54,6 +54,7 @@ struct SmemCtrl {
 };
 static_assert(sizeof(SmemCtrl) <= 512, "SmemCtrl must fit below the staged stage descriptor");
 static_assert(512 + sizeof(Stage) <= 1024, "stage descriptor must fit below the program caches");
+static_assert(sizeof(Stage) % 16 == 0 && sizeof(Addr) % 8 == 0, "staged with vector copies");
 
 // debug timeline mark k of the current stage (CTA 0 only; the calling thread decides who marks),
 // plus a per-CTA copy of marks 0..3 at prof[9*nst + 1 + (stage*kProfCtas + cta)*4 + k]
@@ -160,6 +161,44 @@ struct Vec {
   float x[W];
 };
 
+// ---- shared-memory tensor cache (§6.5; placement decided on the host by an LRU
+// scan, host/lower.cpp tensor_cache).  Every stage that touches a cached tensor is a row-block stage
+// with the same rows and row-block size, so the CTA that deposits row r of the tensor is the CTA that
+// reads it back; the stages are separated by at least a __syncthreads.
+extern __shared__ __align__(1024) char g_dyn_smem[];
+__device__ __forceinline__ float* cache_elem(const Addr& A, int64_t r, int64_t c) {
+  float* base = reinterpret_cast<float*>((((uintptr_t)g_dyn_smem + 1023) & ~(uintptr_t)1023) + EXEC_SMEM);
+  const uint32_t rb = (uint32_t)r / (uint32_t)A.crb;
+  const uint32_t it = rb / gridDim.x;
+  return base + (A.cache - 1) + ((size_t)it * A.crb + (uint32_t)r - rb * (uint32_t)A.crb) * (size_t)A.rs + (size_t)c * A.cs;
+}
+template <int W>
+__device__ __forceinline__ void cache_ld(const Addr& A, int64_t r, int64_t c0, int nvalid, float* v) {
+  const float* q = cache_elem(A, r, c0);
+  if (W == 8 && A.cs == 1 && nvalid == 8 && ((uintptr_t)q & 15) == 0) {
+    const float4 a = reinterpret_cast<const float4*>(q)[0], b = reinterpret_cast<const float4*>(q)[1];
+    v[0] = a.x; v[1 % W] = a.y; v[2 % W] = a.z; v[3 % W] = a.w; v[4 % W] = b.x; v[5 % W] = b.y; v[6 % W] = b.z; v[7 % W] = b.w;
+    return;
+  }
+#pragma unroll
+  for (int j = 0; j < W; ++j) v[j] = j < nvalid ? q[(int64_t)j * A.cs] : 0.f;
+}
+template <int W>
+__device__ __forceinline__ void cache_st(const Addr& A, int64_t r, int64_t c0, int nvalid, const float* v) {
+  float* q = cache_elem(A, r, c0);
+  if (W == 8 && A.cs == 1 && nvalid == 8 && ((uintptr_t)q & 15) == 0) {
+    float u[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) u[j] = A.dtype ? __uint_as_float((uint32_t)f2bf(v[j % W]) << 16) : v[j % W];
+    reinterpret_cast<float4*>(q)[0] = make_float4(u[0], u[1], u[2], u[3]);
+    reinterpret_cast<float4*>(q)[1] = make_float4(u[4], u[5], u[6], u[7]);
+    return;
+  }
+#pragma unroll
+  for (int j = 0; j < W; ++j)   // rounded as a global round trip would round it
+    if (j < nvalid) q[(int64_t)j * A.cs] = A.dtype ? __uint_as_float((uint32_t)f2bf(v[j]) << 16) : v[j];
+}
+
 // The element-access helpers and the unary math exist once each (out of line): with everything
 // inlined the kernel was 1.3 MB of SASS and every stage ran from a cold instruction cache.
 template <int W>
@@ -202,7 +241,7 @@ __device__ __noinline__ Vec<W> ld_vec_impl(const Params& P, const Addr& A, int64
 // Inline fast paths (contiguous vector / row broadcast) so that independent loads of a chunk are
 // all in flight together; only the generic per-element gather is out of line.
 template <int W>
-__device__ __forceinline__ void ld_vec(const Params& P, const Addr& A, int64_t r, int64_t c0, int nvalid, float* v) {
+__device__ __forceinline__ void ld_vec_g(const Params& P, const Addr& A, int64_t r, int64_t c0, int nvalid, float* v) {
   const int64_t o = contig_off<W>(P, A, r, c0, nvalid);
   if (W == 8 && o >= 0 && A.dtype == 0 && (o & 3) == 0) {
     const float4* q = reinterpret_cast<const float4*>((const float*)addr_ptr(P, A) + o);
@@ -231,6 +270,18 @@ __device__ __forceinline__ void ld_vec(const Params& P, const Addr& A, int64_t r
   Vec<W> t = ld_vec_impl<W>(P, A, r, c0, nvalid);
 #pragma unroll
   for (int j = 0; j < W; ++j) v[j] = t.x[j];
+}
+
+// a cached tensor is read from shared memory; a filling load (the tensor's first use in the launch)
+// reads global memory and deposits whole chunks (the W = 1 row-start probe of a shifted reduction does not)
+template <int W>
+__device__ __forceinline__ void ld_vec(const Params& P, const Addr& A, int64_t r, int64_t c0, int nvalid, float* v) {
+  if (A.cache && !(A.cmode & CM_FILL)) {
+    cache_ld<W>(A, r, c0, nvalid, v);
+    return;
+  }
+  ld_vec_g<W>(P, A, r, c0, nvalid, v);
+  if (W == CHUNK && A.cache) cache_st<W>(A, r, c0, nvalid, v);
 }
 
 template <int W>
@@ -268,6 +319,10 @@ __device__ __noinline__ void st_vec_impl(const Params& P, const Addr& A, int64_t
 
 template <int W>
 __device__ __forceinline__ void st_vec(const Params& P, const Addr& A, int64_t r, int64_t c0, int nvalid, const float* v) {
+  if (A.cache) {
+    cache_st<W>(A, r, c0, nvalid, v);
+    if (A.cmode & CM_NOSTORE) return;
+  }
   const int64_t o = contig_off<W>(P, A, r, c0, nvalid);
   if (W == 8 && o >= 0 && A.dtype == 0 && (o & 3) == 0) {
     float4* q = reinterpret_cast<float4*>((float*)addr_ptr(P, A) + o);
@@ -734,6 +789,23 @@ __device__ __noinline__ void run_ew(const Params& P, const Stage& st, char* smem
   const int64_t cpr = (st.cols + CHUNK - 1) / CHUNK;
   const int64_t total = (int64_t)st.rows * cpr;
   float red[MAX_RED] = {0.f, 0.f, 0.f, 0.f};
+  if (st.rblk > 0) {   // row-block ownership (CTA-local dependencies with the launch's REDUCE stages)
+    const int64_t per = (int64_t)st.rblk * cpr;
+    for (int64_t rb = blockIdx.x; rb * st.rblk < st.rows; rb += gridDim.x) {
+      const int64_t n = min(per, total - rb * per);
+      for (int64_t i = threadIdx.x; i < n; i += kThreads) {
+        const int64_t t = rb * per + i;
+        const int64_t r = t / cpr, c0 = (t % cpr) * CHUNK;
+        const int nv = (int)((st.cols - c0) < CHUNK ? (st.cols - c0) : CHUNK);
+        float acc[CHUNK] = {0, 0, 0, 0, 0, 0, 0, 0};
+        run_prog<CHUNK>(P, G, r, c0, nv, acc, red);
+        flush_reds(P, G, r, red);
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) mark(P, ctrl_of(smem), 2);
+    return;
+  }
   for (int64_t t = (int64_t)blockIdx.x * kThreads + threadIdx.x; t < total; t += (int64_t)gridDim.x * kThreads) {
     int64_t r = t / cpr;
     int64_t c0 = (t % cpr) * CHUNK;
@@ -758,13 +830,9 @@ __device__ __noinline__ void run_reduce(const Params& P, const Stage& st, char* 
   const Prog post = cached_prog(smem, 1);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   float red[MAX_RED] = {0.f, 0.f, 0.f, 0.f};
-  const int chunks = (st.cols + CHUNK - 1) / CHUNK;
-  int G = 32;
-  if (chunks <= 16) {
-    G = 1;
-    while (G < chunks) G <<= 1;
-  }
-  const int rpw = 32 / G;                      // rows per warp
+  // the host fixed the row-block size (Stage.rblk = 8 warps x 32/G rows, G = lanes per row)
+  const int rpw = st.rblk / 8;                 // rows per warp
+  const int G = 32 / rpw;
   const int sub = lane / G, gl = lane % G;     // row slot within the warp, lane within the group
   const int64_t rows_per_cta = 8 * rpw;
   for (int64_t ob = (int64_t)blockIdx.x * rows_per_cta + warp * rpw; ob < st.rows; ob += (int64_t)gridDim.x * rows_per_cta) {
@@ -1408,33 +1476,34 @@ __global__ void __launch_bounds__(kThreads, 1) souffle_exec_kernel(const __grid_
 }
 
 cudaError_t exec_launch(const Params& prm, int grid, int smem, bool cooperative, cudaStream_t s) {
+  // smem = the launch's working area (EXEC_SMEM) + its tensor-cache units; +1024 for the alignment
+  constexpr int kMaxDyn = EXEC_SMEM + 1024 + EXEC_CACHE_FLOATS * 4;
+  static_assert(kMaxDyn <= 227 * 1024, "exceeds the opt-in shared memory per block");
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(souffle_exec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         EXEC_SMEM + 1024);
+    cudaError_t e = cudaFuncSetAttribute(souffle_exec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDyn);
     if (e != cudaSuccess) return e;
     attr = true;
   }
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(kThreads);
-  cfg.dynamicSmemBytes = EXEC_SMEM + 1024;
+  cfg.dynamicSmemBytes = (smem > EXEC_SMEM ? smem : EXEC_SMEM) + 1024;
   cfg.stream = s;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeCooperative;
   at[0].val.cooperative = cooperative ? 1 : 0;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  (void)smem;
   return cudaLaunchKernelEx(&cfg, souffle_exec_kernel, prm);
 }
 
 cudaError_t exec_max_active(int smem, int* blocks) {
-  cudaError_t e = cudaFuncSetAttribute(souffle_exec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       EXEC_SMEM + 1024);
+  constexpr int kMaxDyn = EXEC_SMEM + 1024 + EXEC_CACHE_FLOATS * 4;
+  cudaError_t e = cudaFuncSetAttribute(souffle_exec_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxDyn);
   if (e != cudaSuccess) return e;
-  (void)smem;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, souffle_exec_kernel, kThreads, EXEC_SMEM + 1024);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks, souffle_exec_kernel, kThreads,
+                                                       (smem > EXEC_SMEM ? smem : EXEC_SMEM) + 1024);
 }
 
 }  // namespace souffle

@@ -10,8 +10,7 @@
 //          every tag carries this run's step (one round trip = readiness + data; no grid barrier,
 //          no fence; the wavefront is L + T - 1 = 109 cells deep)
 //   GEMV   gates = [W_ih | W_hh] [x_t ; h_{t-1}] on CUDA cores, bf16 (or fp32) weights x fp32
-//          activations, fp32 accumulation (activations are never rounded: SURVEY §8(c)); the 16
-//          warps split K (chunk-major weights, conflict-free), partials summed in warp order
+//          activations, fp32 accumulation (activations are never rounded: SURVEY §8(c))
 //   cell   i, f, o = sigmoid, g = tanh; c = f c + i g; h = o tanh(c)  (torch.nn.LSTM semantics)
 //   publish h(l, t) for the 32 units as (value, tag) 64-bit words
 #include <cuda_bf16.h>
@@ -32,6 +31,24 @@ __device__ __forceinline__ float tanh_f(float x) {
   return copysignf(__fdividef(1.f - t, 1.f + t), x);
 }
 
+// 8 consecutive weights of row r (smem) as fp32
+template <bool F32>
+__device__ __forceinline__ void wload8(const char* w, int K, int r, int g, float* o) {
+  if constexpr (F32) {
+    const float4* p = reinterpret_cast<const float4*>(w) + ((int64_t)r * K + 8 * g) / 4;
+    const float4 a = p[0], b = p[1];
+    o[0] = a.x; o[1] = a.y; o[2] = a.z; o[3] = a.w; o[4] = b.x; o[5] = b.y; o[6] = b.z; o[7] = b.w;
+  } else {
+    const uint4 a = *reinterpret_cast<const uint4*>(reinterpret_cast<const uint16_t*>(w) + (int64_t)r * K + 8 * g);
+    const uint32_t u[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      o[2 * j] = __uint_as_float(u[j] << 16);
+      o[2 * j + 1] = __uint_as_float(u[j] & 0xFFFF0000u);
+    }
+  }
+}
+
 template <bool F32>
 __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_constant__ LstmParams P) {
   extern __shared__ __align__(16) char smem[];
@@ -43,27 +60,22 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
   const LstmLayer& Ly = P.layers[l];
   const int I = Ly.in_dim, K = I + H;
   constexpr int ES = F32 ? 4 : 2;
-  // weights chunk-major: 16-byte chunk (kc, r) = elements [kc * EPC, kc * EPC + EPC) of gate row r at
-  // byte (kc * LSTM_ROWS + r) * 16, so the lanes of a warp (consecutive rows, one chunk) read 512
-  // contiguous bytes -- conflict-free
-  constexpr int EPC = 16 / ES;   // elements per chunk
-  char* w = smem;                                                        // [K_max / EPC][128][16 B]
+  char* w = smem;                                                        // [128][Kst] weights
   float* xh = reinterpret_cast<float*>(smem + (size_t)LSTM_ROWS * Kst * ES);   // [Kst]  [x_t ; h_{t-1}]
   float* gates = xh + Kst;                                               // [128]
   float* bias = gates + LSTM_ROWS;                                       // [128] b_ih + b_hh
-  float* part = bias + LSTM_ROWS;                                        // [16 warps][128] GEMV partials
 
   // ---- weights of this CTA's 128 gate rows -> shared memory (once for all T steps)
   {
-    const int nch = K / EPC;
-    for (int e = tid; e < LSTM_ROWS * nch; e += LSTM_THREADS) {
-      const int r = e % LSTM_ROWS, kc = e / LSTM_ROWS;
-      if (r >= R) continue;
+    const int vpr = K * ES / 16;   // 16-byte vectors per row
+    for (int e = tid; e < LSTM_ROWS * vpr; e += LSTM_THREADS) {
+      const int r = e / vpr, v = e % vpr;
+      if (r >= R) break;
       const int grow = (r / nu) * H + u0 + (r % nu);
-      const int col = kc * EPC;   // a chunk never straddles [W_ih | W_hh] (I % EPC == 0)
+      const int col = v * 16 / ES;   // first element of this vector
       const char* src = col < I ? (const char*)Ly.W + ((int64_t)grow * I + col) * ES
                                 : (const char*)Ly.U + ((int64_t)grow * H + (col - I)) * ES;
-      *reinterpret_cast<uint4*>(w + ((int64_t)kc * LSTM_ROWS + r) * 16) = __ldg(reinterpret_cast<const uint4*>(src));
+      *reinterpret_cast<uint4*>(w + ((int64_t)r * Kst + col) * ES) = __ldg(reinterpret_cast<const uint4*>(src));
     }
     for (int r = tid; r < R; r += LSTM_THREADS) {
       const int grow = (r / nu) * H + u0 + (r % nu);
@@ -116,52 +128,50 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
     }
     __syncthreads();
     stamp(t, 1);
-    // ---- gates: warp w takes a contiguous range of K chunks for ALL rows, lane j rows j, j+32, j+64,
-    // j+96 (all 16 warps busy, no shuffles); the 16 per-warp partial sums of a row are then added in
-    // warp order (deterministic) by one thread per row
-    {
-      const int nch = K / EPC, cpw = (nch + 15) / 16;
-      const int kc0 = warp * cpw, kc1 = min(nch, kc0 + cpw);
-      float acc[4] = {0.f, 0.f, 0.f, 0.f};
-      for (int kc = kc0; kc < kc1; ++kc) {
-        float xv[EPC];
-        if constexpr (F32) {
-          const float4 xa = *reinterpret_cast<const float4*>(xh + 4 * kc);
-          xv[0] = xa.x; xv[1] = xa.y; xv[2] = xa.z; xv[3] = xa.w;
-        } else {
-          const float4 xa = *reinterpret_cast<const float4*>(xh + 8 * kc);
-          const float4 xb = *reinterpret_cast<const float4*>(xh + 8 * kc + 4);
-          xv[0] = xa.x; xv[1] = xa.y; xv[2] = xa.z; xv[3] = xa.w; xv[4] = xb.x; xv[5] = xb.y; xv[6] = xb.z; xv[7] = xb.w;
-        }
-        const uint4* wc = reinterpret_cast<const uint4*>(w + (int64_t)kc * LSTM_ROWS * 16);
+    // ---- gates: warp w computes rows RPW*w ..; lanes split the K columns in groups of 8 (warps
+    // beyond the CTA's 4 nu rows skip: the smem weight reads are the step's bound)
+    if (warp * 8 < R) {
+      constexpr int RPW = LSTM_ROWS / (LSTM_THREADS / 32);   // rows per warp (8 with 16 warps)
+      static_assert(RPW == 8, "reduction below assumes 8 rows per warp");
+      float acc[RPW];
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int r = lane + 32 * i;
-          if (r < R) {
-            const uint4 q = wc[r];
-            const uint32_t u[4] = {q.x, q.y, q.z, q.w};
-            if constexpr (F32) {
+      for (int i = 0; i < RPW; ++i) acc[i] = 0.f;
+      const int ng = K / 8;
+      for (int g = lane; g < ng; g += 32) {
+        const float4 xa = *reinterpret_cast<const float4*>(xh + 8 * g);
+        const float4 xb = *reinterpret_cast<const float4*>(xh + 8 * g + 4);
+        const float xv[8] = {xa.x, xa.y, xa.z, xa.w, xb.x, xb.y, xb.z, xb.w};
+        float wv[RPW][8];
 #pragma unroll
-              for (int e = 0; e < 4; ++e) acc[i] = fmaf(__uint_as_float(u[e]), xv[e], acc[i]);
-            } else {
+        for (int i = 0; i < RPW; ++i) wload8<F32>(w, Kst, warp * RPW + i, g, wv[i]);
 #pragma unroll
-              for (int e = 0; e < 4; ++e) {
-                acc[i] = fmaf(__uint_as_float(u[e] << 16), xv[2 * e], acc[i]);
-                acc[i] = fmaf(__uint_as_float(u[e] & 0xFFFF0000u), xv[2 * e + 1], acc[i]);
-              }
-            }
-          }
-        }
+        for (int i = 0; i < RPW; ++i)
+#pragma unroll
+          for (int e = 0; e < 8; ++e) acc[i] = fmaf(wv[i][e], xv[e], acc[i]);
       }
+      // transpose-reduce 8 row sums over the 32 lanes (4 + 2 + 1 + 2 shuffles)
+      float v4[4];
+      const bool b4 = lane & 16;
 #pragma unroll
-      for (int i = 0; i < 4; ++i) part[warp * LSTM_ROWS + lane + 32 * i] = acc[i];
-      __syncthreads();
-      if (tid < R) {
-        float g = 0.f;
-#pragma unroll
-        for (int k = 0; k < LSTM_THREADS / 32; ++k) g += part[k * LSTM_ROWS + tid];
-        gates[tid] = g;
+      for (int i = 0; i < 4; ++i) {
+        const float send = b4 ? acc[i] : acc[i + 4];
+        const float keep = b4 ? acc[i + 4] : acc[i];
+        v4[i] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
       }
+      float v2[2];
+      const bool b3 = lane & 8;
+#pragma unroll
+      for (int i = 0; i < 2; ++i) {
+        const float send = b3 ? v4[i] : v4[i + 2];
+        const float keep = b3 ? v4[i + 2] : v4[i];
+        v2[i] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+      }
+      const bool b2 = lane & 4;
+      float v1 = (b2 ? v2[1] : v2[0]) + __shfl_xor_sync(0xffffffffu, b2 ? v2[0] : v2[1], 4);
+      v1 += __shfl_xor_sync(0xffffffffu, v1, 2);
+      v1 += __shfl_xor_sync(0xffffffffu, v1, 1);
+      const int r = 4 * ((lane >> 4) & 1) + 2 * ((lane >> 3) & 1) + ((lane >> 2) & 1);
+      if ((lane & 3) == 0) gates[warp * RPW + r] = v1;
     }
     __syncthreads();
     stamp(t, 2);
@@ -200,7 +210,7 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
 }  // namespace lstm
 
 size_t lstm_smem_bytes(int K_max, int w_f32) {
-  return (size_t)LSTM_ROWS * K_max * (w_f32 ? 4 : 2) + (size_t)(K_max + 2 * LSTM_ROWS + (LSTM_THREADS / 32) * LSTM_ROWS) * 4;
+  return (size_t)LSTM_ROWS * K_max * (w_f32 ? 4 : 2) + (size_t)(K_max + 2 * LSTM_ROWS) * 4;
 }
 
 cudaError_t lstm_launch(const LstmParams& prm, int grid, cudaStream_t s) {

@@ -216,6 +216,41 @@ def random_spec(seed: int, n_ops: int = 12, dim_choices=(2, 3, 4, 5)) -> dict:
     return {"nodes": nodes, "outputs": [len(nodes) - 1]}
 
 
+def random_rowwise_spec(seed: int, n_ops: int = 14) -> dict:
+    """Random row-wise TE program over one [R, C] domain (structure only): chains of row reductions
+    (sum / max / mean, keepdim) and elementwise ops that combine [R, C] tensors with the [R, 1]
+    statistics -- the LayerNorm / softmax shape of dependence that the generic executor runs as
+    reduction and elementwise stages over the same rows (tensor reuse, §6.5).  R spans several row
+    blocks per CTA; C includes ragged widths (not a multiple of 8)."""
+    r = rng(seed)
+    nodes = []
+
+    def add(node):
+        nodes.append(node)
+        return len(nodes) - 1
+
+    R = int(r.choice([200, 300, 1000, 4000]))
+    C = int(r.choice([8, 24, 49, 64, 130]))
+    full = [add(dict(op="placeholder", shape=[R, C], dtype="f32", const=0)) for _ in range(int(r.choice([1, 2, 3])))]
+    stats = []
+    for _ in range(n_ops):
+        kind = r.choice(["red", "red", "bin_stat", "bin_stat", "bin", "un"])
+        src = int(r.choice(full))
+        if kind == "red":
+            fn = str(r.choice(["sum", "max", "mean"]))
+            stats.append(add(dict(op="reduce", fn=fn, **{"in": src}, axis=1, keepdim=1)))
+        elif kind == "bin_stat" and stats:
+            fn = str(r.choice(["sub", "mul", "add"]))
+            full.append(add(dict(op="ew", fn=fn, **{"in": [src, int(r.choice(stats))]}, scalar=0.0)))
+        elif kind == "bin" and len(full) > 1:
+            other = int(r.choice([i for i in full if i != src]))
+            full.append(add(dict(op="ew", fn=str(r.choice(["add", "mul", "max"])), **{"in": [src, other]}, scalar=0.0)))
+        else:
+            full.append(add(dict(op="ew", fn=str(r.choice(["tanh", "sigmoid", "neg"])), **{"in": [src]}, scalar=0.0)))
+    outs = [full[-1]] + ([stats[-1]] if stats else [])
+    return {"nodes": nodes, "outputs": outs}
+
+
 def spec_inputs(spec: dict, seed: int, integer: bool = False) -> dict:
     """Seeded values for every placeholder of a spec (dict id -> float32 array in storage dtype)."""
     out = {}

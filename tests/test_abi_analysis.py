@@ -13,6 +13,7 @@ from oracle import graphs as og
 from oracle import te
 from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
 from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+import synth.swin as synth_swin
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
@@ -245,3 +246,49 @@ def test_swin_pattern_matches_and_skips_generic_lowering():
     # fp32 GEMMs are outside the pattern (bf16 tcgen05 operands): generic path
     g, *_ = M.swin(S.SWIN_TINY)
     assert "pattern swin: not used" in g.partition(L.device_b200()).describe()
+
+
+def _cache_stats(plan):
+    d = plan.describe()
+    m = re.search(r"tensor cache: (\d+) tensor.*?(\d+) hit.*?(\d+) LRU.*?(\d+) global", d)
+    return [int(x) for x in m.groups()] if m else None
+
+
+def test_tensor_reuse_plan_swin_generic():
+    """§6.5 tensor reuse in the generic lowering: LayerNorm / softmax reductions and their
+    elementwise consumers share row blocks, so their dependencies need no grid barrier and the re-read
+    activations are served from the shared-memory cache.  The analysis itself does not change."""
+    g = M.swin(dict(synth_swin.SWIN_TINY, batch=1))[0]
+    on = g.partition(L.device_b200(), flags=L.FLAG_NO_PATTERN)
+    off = g.partition(L.device_b200(), flags=L.FLAG_NO_PATTERN | L.FLAG_NO_PREFETCH)
+    assert on.assignment() == off.assignment() and on.bfs_order() == off.bfs_order()
+    assert on.exec_info()["stages"] == off.exec_info()["stages"]
+    assert on.exec_info()["barriers"] < off.exec_info()["barriers"]
+    tensors, hits, _, _ = _cache_stats(on)
+    assert tensors > 0 and hits >= tensors
+    assert _cache_stats(off) is None
+    assert _cache_stats(g.partition(L.device_b200(), flags=L.FLAG_UNFUSED)) is None
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_rowwise_programs_need_no_grid_barrier(seed):
+    """A row-wise program (reductions + elementwise over one [R, C] domain) has only CTA-local
+    dependencies under reuse; without it every reduction consumer waits at a grid barrier."""
+    g = M.from_spec(synth.random_rowwise_spec(seed))
+    on = g.partition(L.device_b200()).exec_info()
+    off = g.partition(L.device_b200(), flags=L.FLAG_NO_PREFETCH).exec_info()
+    assert on["barriers"] == 0
+    assert off["barriers"] >= on["barriers"]
+
+
+def test_tensor_cache_lru_spills_under_small_capacity(monkeypatch):
+    """Capacity 2048 floats holds one Swin-tiny LayerNorm row block: the LRU scan must evict tensors
+    whose readers are still to come (they then read global memory: the spill) and place fewer."""
+    g = M.swin(dict(synth_swin.SWIN_TINY, batch=1))[0]
+    full = _cache_stats(g.partition(L.device_b200(), flags=L.FLAG_NO_PATTERN))
+    monkeypatch.setenv("SOUFFLE_CACHE_FLOATS", "2048")
+    small = _cache_stats(g.partition(L.device_b200(), flags=L.FLAG_NO_PATTERN))
+    assert full[2] == 0 and small[2] > 0
+    assert small[1] < full[1]
+    monkeypatch.setenv("SOUFFLE_CACHE_FLOATS", "0")
+    assert _cache_stats(g.partition(L.device_b200(), flags=L.FLAG_NO_PATTERN))[:2] == [0, 0]

@@ -77,6 +77,41 @@ def test_random_programs_generic_path(seed):
             assert rel_err(y, ref[o]) <= 1e-4, (flags, plan.describe())
 
 
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("cache", [None, "4096", "2048"])
+def test_rowwise_programs_tensor_cache(seed, cache, monkeypatch, record_err):
+    """§6.5 tensor reuse: row-wise reduction / elementwise programs whose stages hand
+    each row block to the same CTA -- CTA-local dependencies without grid barriers, tensors kept in
+    the shared-memory cache.  cache = SOUFFLE_CACHE_FLOATS: the default capacity, then capacities
+    small enough that the LRU scan evicts tensors with readers still to come (spills to global) or
+    cannot place them at all.  NO_PREFETCH turns reuse off; NO_GLOBAL_SYNC splits at the barriers."""
+    if cache:
+        monkeypatch.setenv("SOUFFLE_CACHE_FLOATS", cache)
+    spec = synth.random_rowwise_spec(seed)
+    ins = synth.spec_inputs(spec, seed)
+    g = M.from_spec(spec)
+    ref = te.evaluate(spec, ins)
+    for flags in (0, L.FLAG_NO_PREFETCH, L.FLAG_NO_GLOBAL_SYNC):
+        outs, plan = run(g, ins, spec["outputs"], flags)
+        d = plan.describe()
+        if flags & L.FLAG_NO_PREFETCH:
+            assert "tensor cache" not in d
+        for o, y in zip(spec["outputs"], outs):
+            record_err(rel_err(y, ref[o]), 1e-4, flags=flags, cache=cache,
+                       plan=[ln for ln in d.splitlines() if ln.startswith(("plan:", "tensor cache"))])
+
+
+def test_tensor_cache_spills_are_exercised(monkeypatch):
+    """The forced-capacity cases above really evict tensors with pending readers (host plan only)."""
+    ev = 0
+    for cache in ("4096", "2048"):
+        monkeypatch.setenv("SOUFFLE_CACHE_FLOATS", cache)
+        for seed in range(12):
+            d = M.from_spec(synth.random_rowwise_spec(seed)).partition(L.device_query(0)).describe()
+            ev += int(d.split("hit(s), ")[1].split(" LRU")[0])
+    assert ev >= 3
+
+
 @pytest.mark.parametrize("flags", [0, L.FLAG_UNFUSED, L.FLAG_NO_LN_REWRITE, L.FLAG_NO_VERTICAL])
 def test_bert_tiny_fp32(flags):
     cfg = synth.BERT_TINY

@@ -39,9 +39,15 @@ def _run(cfg, flags=0, bf16=False):
 
 
 @pytest.mark.parametrize("batch", [1, 2])
-@pytest.mark.parametrize("flags", [0, L.FLAG_UNFUSED])
-def test_swin_tiny_fp32(batch, flags):
+@pytest.mark.parametrize("flags,cache", [(0, None), (L.FLAG_UNFUSED, None), (L.FLAG_NO_PREFETCH, None), (0, "2048")])
+def test_swin_tiny_fp32(batch, flags, cache, monkeypatch):
+    """Generic executor.  cache: SOUFFLE_CACHE_FLOATS -- 2048 floats hold one LayerNorm row block of
+    x at a time, so the LRU scan spills tensors whose readers are still to come (§6.5)."""
+    if cache:
+        monkeypatch.setenv("SOUFFLE_CACHE_FLOATS", cache)
     got, again, ref, plan = _run(dict(S.SWIN_TINY, batch=batch), flags)
+    if cache:
+        assert "0 LRU eviction" not in plan.describe()
     assert rel_err(got, ref) <= 1e-4, plan.describe()[:2000]
     assert rel_err(again, ref) <= 1e-4
 
