@@ -7,6 +7,8 @@ nvidia-smi > gpurun_out/r02_nvsmi.txt 2>&1
 python -c "from paper_conf_asplos_xiazswwyfc24_b200.build import build; build()" > gpurun_out/build.log 2>&1
 timeout 1500 python -m pytest tests -q -m gpu > gpurun_out/r02_pytest_gpu.txt 2>&1
 echo "rc=$?" >> gpurun_out/r02_pytest_gpu.txt
+timeout 600 python -c "import __graft_entry__ as e; e.smoke()" > gpurun_out/r02_smoke.txt 2>&1
+echo "rc=$?" >> gpurun_out/r02_smoke.txt
 timeout 1500 python bench.py > gpurun_out/r02_bench.json 2> gpurun_out/r02_bench.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/r02_launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-v0 --no-models > gpurun_out/r02_ncu_launch.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:bert_kernel -s 1 -c 1 -o gpurun_out/r02_prof_bert python tools/run_once.py bert_base 0 0 2 > gpurun_out/r02_ncu_full.log 2>&1
