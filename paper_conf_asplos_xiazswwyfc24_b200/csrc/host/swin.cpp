@@ -456,6 +456,10 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
       if (N % bn == 0 && mt * (N / bn) >= nsm) { g.BN = bn; break; }
     }
     if (g.BN == 64 && N % 64) g.BN = N % 128 == 0 ? 128 : 256;
+    if (const char* e = std::getenv("SOUFFLE_SWIN_BN")) {   // tile studies: force the N tile where it divides N
+      const int bn = std::atoi(e);
+      if ((bn == 64 || bn == 128 || bn == 256) && N % bn == 0) g.BN = bn;
+    }
     g.stages = g.BN == 256 ? 4 : g.BN == 128 ? 6 : 8;
     const int tiles = (int)(N / g.BN * mt);
     g.splits = 1;
