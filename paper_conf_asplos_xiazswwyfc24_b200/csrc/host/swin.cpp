@@ -456,6 +456,11 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
       if (N % bn == 0 && mt * (N / bn) >= nsm) { g.BN = bn; break; }
     }
     if (g.BN == 64 && N % 64) g.BN = N % 128 == 0 ? 128 : 256;
+    // narrow outputs (proj, fc2, patch merge: 256 <= N <= 1024) take 128-wide tiles: with 256 their tile count
+    // lands just above one wave (b64: 196 tiles on 148 SMs), with 64 the residual epilogue's row
+    // traffic per MMA doubles -- measured at b8 / b64 (profiles/r02_swin_bn_study.txt); small M keeps
+    // the split-K policy (batch 1 measured slower with 128)
+    if (N >= 256 && N <= 1024 && N % 128 == 0 && mt >= 8 && g.BN != 128 && !std::getenv("SOUFFLE_SWIN_BN_OLD")) g.BN = 128;
     if (const char* e = std::getenv("SOUFFLE_SWIN_BN")) {   // tile studies: force the N tile where it divides N
       const int bn = std::atoi(e);
       if ((bn == 64 || bn == 128 || bn == 256) && N % bn == 0) g.BN = bn;
