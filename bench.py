@@ -141,9 +141,25 @@ def cpu_baseline(budget_s=15.0):
         if el >= budget_s or n >= 24:
             break
     inf_s = (n / NL) / el
-    return {"value": inf_s, "unit": "inferences/s", "cores": os.cpu_count(), "kind": "oracle",
-            "sample": f"{n} BERT-base encoder layers (= {n / NL:.2f} inferences) of the fp64 numpy oracle "
-                      f"(bf16-operand emulation), {el:.1f} s wall, OpenBLAS threads = host cores"}
+    out = {"value": inf_s, "unit": "inferences/s", "cores": os.cpu_count(), "kind": "oracle",
+           "sample": f"{n} BERT-base encoder layers (= {n / NL:.2f} inferences) of the fp64 numpy oracle "
+                     f"(bf16-operand emulation), {el:.1f} s wall, OpenBLAS threads = host cores"}
+    try:   # the same oracle on ONE core (BLAS pool limited to one thread)
+        from threadpoolctl import threadpool_limits
+        with threadpool_limits(limits=1):
+            step()
+            n1, t1 = 0, time.perf_counter()
+            while True:
+                step()
+                n1 += 1
+                el1 = time.perf_counter() - t1
+                if el1 >= budget_s / 2 or n1 >= 12:
+                    break
+        out["single_thread"] = {"value": (n1 / NL) / el1, "unit": "inferences/s", "cores": 1,
+                                "sample": f"{n1} encoder layers, {el1:.1f} s wall, BLAS threads = 1"}
+    except Exception as e:  # noqa: BLE001 -- a missing threadpoolctl only drops the extra figure
+        out["single_thread"] = {"unavailable": str(e)[:120]}
+    return out
 
 
 def run_reference(args):
