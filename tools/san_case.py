@@ -1,5 +1,7 @@
 """One small launch of a kernel family, checked against the oracle (for compute-sanitizer runs).
-usage: python tools/san_case.py bert_small | swin_small | generic_tiny"""
+usage: python tools/san_case.py bert_small | swin_small | generic_tiny | rowwise | swin_generic
+(rowwise / swin_generic / generic_tiny exercise the generic executor's row-block stages and tensor cache;
+SOUFFLE_CACHE_FLOATS=2048 forces LRU spills)"""
 import os
 import sys
 
@@ -25,8 +27,18 @@ if which in ("bert_small", "generic_tiny"):
     s = session(g, plan, og.bert_feed(gX, gpl, x, w), [gy])
     s.run()
     out = s.result(gy)
+elif which == "rowwise":
+    spec = synth.random_rowwise_spec(0)
+    ins = synth.spec_inputs(spec, 0)
+    g = M.from_spec(spec)
+    plan = g.partition(L.device_query(0))
+    s = session(g, plan, ins, spec["outputs"])
+    s.run()
+    o = spec["outputs"][0]
+    out, ref = s.result(o), te.evaluate(spec, ins)[o]
 else:
-    cfg = dict(SW.SWIN_TINY, embed=128, heads=(4, 8), gemm_dtype="bf16")
+    cfg = dict(SW.SWIN_TINY, embed=128, heads=(4, 8), gemm_dtype="bf16") if which == "swin_small" else \
+        dict(SW.SWIN_TINY, batch=1)
     P = SW.swin_params(cfg)
     fv = SW.swin_feed_values(cfg, P)
     img = SW.swin_input(cfg)
@@ -38,5 +50,6 @@ else:
     s.run()
     out = s.result(gy)
     spec, on, ox, oy = og.swin(cfg)
-    ref = te.evaluate(spec, feed, bf16_operands=True)[oy]
-print(which, plan.describe().splitlines()[0][:100], "max abs err", float(np.abs(out - ref).max()))
+    ref = te.evaluate(spec, feed, bf16_operands=cfg.get("gemm_dtype") == "bf16")[oy]
+info = [ln for ln in plan.describe().splitlines() if ln.startswith(("plan:", "tensor cache"))]
+print(which, info, "max abs err", float(np.abs(out - ref).max()))
