@@ -3,7 +3,8 @@ under the optimisation ladder, through the same C ABI (median of L2-flushed runs
   V0  unfused: one kernel per TE                      (SOUFFLE_FLAG_UNFUSED)
   V1  + horizontal transformation                     (NO_VERTICAL | NO_GLOBAL_SYNC | NO_PATTERN)
   V2  + vertical transformation                       (NO_GLOBAL_SYNC | NO_PATTERN)
-  V3  + global synchronisation: one launch per SP     (NO_PATTERN: generic executor, everything on)
+  V3  + global synchronisation: one launch per SP     (NO_PATTERN | NO_PREFETCH: generic executor)
+  V3r + §6.5 tensor reuse in the generic executor     (NO_PATTERN: row-block stages, LRU smem cache)
   V4  + the model's pattern kernel (persistent, cross-stage weight prefetch / on-chip weights)
 usage: python tools/ablation.py [models...]   (bert lstm mmoe swin) -> JSON lines on stdout"""
 import json
@@ -23,7 +24,8 @@ from paper_conf_asplos_xiazswwyfc24_b200 import models as M  # noqa: E402
 from paper_conf_asplos_xiazswwyfc24_b200.session import session  # noqa: E402
 
 VARIANTS = [("V0", L.FLAG_UNFUSED), ("V1", L.FLAG_NO_VERTICAL | L.FLAG_NO_GLOBAL_SYNC | L.FLAG_NO_PATTERN),
-            ("V2", L.FLAG_NO_GLOBAL_SYNC | L.FLAG_NO_PATTERN), ("V3", L.FLAG_NO_PATTERN), ("V4", 0)]
+            ("V2", L.FLAG_NO_GLOBAL_SYNC | L.FLAG_NO_PATTERN), ("V3", L.FLAG_NO_PATTERN | L.FLAG_NO_PREFETCH),
+            ("V3r", L.FLAG_NO_PATTERN), ("V4", 0)]
 
 
 def graph_and_feed(name):
