@@ -271,7 +271,12 @@ void bert_match(const Graph& g, const Analysis& an, const souffle_device_desc& d
     const int kc = bp.H / 64;
     bp.pairs = (!e || std::atoi(e) != 0) && sms % 2 == 0 && kc % 2 == 0;
     if (bp.pairs) {
-      const BertGemmCfg q{32, 2, kc / 2, 3 * bp.H / 32}, f{64, 2, kc / 2, bp.F / 64};
+      int qn = 32, fn = 64;   // N tiles of the pair GEMMs (SOUFFLE_BERT_PAIR_NT=qkv,ffn1 for tile studies)
+      if (const char* t = std::getenv("SOUFFLE_BERT_PAIR_NT")) {
+        int a = 0, b = 0;
+        if (std::sscanf(t, "%d,%d", &a, &b) == 2 && (a == 32 || a == 64) && (b == 32 || b == 64)) { qn = a; fn = b; }
+      }
+      const BertGemmCfg q{qn, 2, kc / 2, (int)(3 * bp.H / qn)}, f{fn, 2, kc / 2, (int)(bp.F / fn)};
       if (q.tiles_n * 2 <= sms && f.tiles_n * 2 <= sms) {
         bp.qkv = q;
         bp.ffn1 = f;
