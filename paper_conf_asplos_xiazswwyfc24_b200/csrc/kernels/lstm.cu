@@ -91,6 +91,10 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
   auto stamp = [&](int t, int k) {   // debug timeline: SM clock cycles (%globaltimer ticks in 256 ns steps)
     if (P.prof && blockIdx.x == P.prof_cta && tid == 0) P.prof[4 * t + k] = (unsigned long long)clock64();
   };
+  // [x_t ; h_{t-1}] is kept split: elements 8g..8g+3 at float4 g, 8g+4..8g+7 at float4 K/8 + g, so the
+  // GEMV lanes (consecutive g) read consecutive float4s (the interleaved layout was 2-way bank-conflicted)
+  const int khalf = K / 2;
+  auto xpos = [&](int k) { return ((k >> 3) << 2) + (k & 3) + ((k & 4) ? khalf : 0); };
   const unsigned gen = *(volatile unsigned*)P.gen;   // written by the previous launch's last CTA
   const unsigned tag0 = gen * (unsigned)(T + 1) + 1u;
   for (int t = 0; t < T; ++t) {
@@ -109,9 +113,9 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
         src[i] = nullptr;
         if (k >= K) continue;
         if (k < I && l == 0) {
-          xh[k] = __ldg(P.X + (int64_t)t * I + k);
+          xh[xpos(k)] = __ldg(P.X + (int64_t)t * I + k);
         } else if (k >= I && t == 0) {
-          xh[k] = __ldg(Ly.h0 + (k - I));
+          xh[xpos(k)] = __ldg(Ly.h0 + (k - I));
         } else {
           src[i] = (k < I) ? P.hbuf + ((int64_t)(l - 1) * T + t) * H + k : P.hbuf + ((int64_t)l * T + t - 1) * H + (k - I);
           want[i] = tag0 + (unsigned)(k < I ? t : t - 1);
@@ -123,7 +127,7 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
         if (src[i] == nullptr) continue;
         while ((unsigned)(w64[i] >> 32) != want[i])   // one single-copy-atomic word: tag in the high half
           asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w64[i]) : "l"(src[i]) : "memory");
-        xh[tid + i * LSTM_THREADS] = __uint_as_float((unsigned)w64[i]);
+        xh[xpos(tid + i * LSTM_THREADS)] = __uint_as_float((unsigned)w64[i]);
       }
     }
     __syncthreads();
@@ -138,8 +142,8 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
       for (int i = 0; i < RPW; ++i) acc[i] = 0.f;
       const int ng = K / 8;
       for (int g = lane; g < ng; g += 32) {
-        const float4 xa = *reinterpret_cast<const float4*>(xh + 8 * g);
-        const float4 xb = *reinterpret_cast<const float4*>(xh + 8 * g + 4);
+        const float4 xa = *reinterpret_cast<const float4*>(xh + 4 * g);
+        const float4 xb = *reinterpret_cast<const float4*>(xh + khalf + 4 * g);
         const float xv[8] = {xa.x, xa.y, xa.z, xa.w, xb.x, xb.y, xb.z, xb.w};
         float wv[RPW][8];
 #pragma unroll
