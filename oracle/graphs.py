@@ -432,3 +432,74 @@ def se_module(cfg):
     y = b.ew("mul", x, g)                      # channel-wise rescale (broadcast over rows)
     b.out(y)
     return b.spec(), dict(x=x, W1=W1, b1=b1, W2=W2, b2=b2), x, y
+
+
+def mbconv(cfg):
+    """EfficientNet MBConv block (the building block of PAPER.md Fig. 5 / 6, L1511-1564; torchvision
+    efficientnet_b0 MBConv in inference form) as a TE program over NHWC, batch 1:
+      a = SiLU(BN(x W_e^T))                      1x1 expand convolution (omitted when expand == 1)
+      d = SiLU(BN(sum_t m_t * roll(a, -o_t) * w_t))[::s, ::s]
+                                                  depthwise k x k convolution, zero padding k // 2: tap t
+                                                  reads a shifted by its offset o_t (a roll TE) and the
+                                                  border mask m_t zeroes what the roll wrapped around
+      d = d * sigmoid(fc2(SiLU(fc1(mean(d)))))    squeeze-and-excitation (se_module)
+      y = BN(d W_p^T) (+ x when stride 1 and cin == cout)
+    BN is the per-channel affine y = x * s + b.  Returns (spec, names, x id, y id)."""
+    d_ = synth_dims(cfg)
+    H, k, s, pad = cfg["hw"], cfg["k"], cfg["stride"], cfg["k"] // 2
+    cin, cout, exp, S = cfg["cin"], cfg["cout"], d_["exp"], d_["squeeze"]
+    Ho = H // s
+    b = SpecBuilder()
+    names = {}
+    x = b.ph((H * H, cin), const=0)
+    a = x
+    if cfg["expand"] != 1:
+        names["We"] = b.ph((exp, cin))
+        a = b.mm(x, names["We"], 1, "f32")
+        names["se"], names["be"] = b.ph((exp,)), b.ph((exp,))
+        a = b.ew("add", b.ew("mul", a, names["se"]), names["be"])
+        a = b.ew("mul", a, b.ew("sigmoid", a))
+    a3 = b.reshape(a, (H, H, exp))
+    acc = None
+    for i in range(k):
+        for j in range(k):
+            t = i * k + j
+            if i == pad and j == pad:
+                term = a3
+            else:
+                r = b._add({"op": "roll", "in": a3, "shifts": [pad - i, pad - j, 0]})   # r[h, w] = a[h + i - pad, w + j - pad]
+                names[f"m{t}"] = b.ph((H, H, 1))
+                term = b.ew("mul", r, names[f"m{t}"])
+            names[f"w{t}"] = b.ph((exp,))
+            term = b.ew("mul", term, names[f"w{t}"])
+            acc = term if acc is None else b.ew("add", acc, term)
+    if s != 1:
+        acc = b.slice(acc, (0, 0, 0), (H, H, exp), (s, s, 1))
+    dd = b.reshape(acc, (Ho * Ho, exp))
+    names["sd"], names["bd"] = b.ph((exp,)), b.ph((exp,))
+    dd = b.ew("add", b.ew("mul", dd, names["sd"]), names["bd"])
+    dd = b.ew("mul", dd, b.ew("sigmoid", dd))
+    p = b.red("mean", dd, 0)
+    names["W1"] = b.ph((S, exp))
+    h = b.mm(p, names["W1"], 1, "f32")
+    names["b1"] = b.ph((S,))
+    h = b.ew("add", h, names["b1"])
+    h = b.ew("mul", h, b.ew("sigmoid", h))
+    names["W2"] = b.ph((exp, S))
+    g = b.mm(h, names["W2"], 1, "f32")
+    names["b2"] = b.ph((exp,))
+    g = b.ew("sigmoid", b.ew("add", g, names["b2"]))
+    dd = b.ew("mul", dd, g)
+    names["Wp"] = b.ph((cout, exp))
+    y = b.mm(dd, names["Wp"], 1, "f32")
+    names["sp"], names["bp"] = b.ph((cout,)), b.ph((cout,))
+    y = b.ew("add", b.ew("mul", y, names["sp"]), names["bp"])
+    if s == 1 and cin == cout:
+        y = b.ew("add", y, x)
+    b.out(y)
+    return b.spec(), names, x, y
+
+
+def synth_dims(cfg):
+    """exp, squeeze of an MBConv config (torchvision: squeeze = max(1, cin // 4))."""
+    return dict(exp=cfg["cin"] * cfg["expand"], squeeze=max(1, cfg["cin"] // 4))

@@ -490,6 +490,12 @@ souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t
       if (barriers) *barriers = 3;
       return;
     }
+    if (P.mb.on) {   // expand, depthwise + pool, pooled, fc1, fc2 + project (+ split-K finish)
+      if (launches) *launches = 1;
+      if (stages) *stages = 5;
+      if (barriers) *barriers = 4;
+      return;
+    }
     if (P.swin.on) {   // one kernel per fused subprogram, replayed as one CUDA graph
       if (launches) *launches = P.swin.launches;
       if (stages) *stages = P.swin.launches;

@@ -10,6 +10,7 @@
 #include "mmoe.h"
 #include "swin.h"
 #include "se.h"
+#include "mbconv.h"
 #include "ir.h"
 
 namespace souffle {
@@ -64,6 +65,7 @@ struct Plan {
   MmoePlan mmoe;                    // pattern lowering (mmoe.on: kernels/mmoe.cu runs the program)
   SwinPlan swin;                    // pattern lowering (swin.on: kernels/swin.cu, one CUDA graph)
   SePlan se;                        // pattern lowering (se.on: kernels/se.cu, EfficientNet M0-M9)
+  MbPlan mb;                        // pattern lowering (mb.on: kernels/mbconv.cu, MBConv blocks M0-M9)
   ~Plan();
 };
 

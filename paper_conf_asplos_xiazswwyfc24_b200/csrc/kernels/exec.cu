@@ -930,17 +930,22 @@ __device__ __noinline__ void run_gemm_simt(const Params& P, const Stage& st, cha
       }
       continue;
     }
-    const int tmi = local / M.tiles_n, tn = local % M.tiles_n;
+    // split-K (few tiles, long K): task = (tile, split); split s accumulates K range [s k_split, ...)
+    const int split = M.splits > 1 ? local % M.splits : 0;
+    const int tl = M.splits > 1 ? local / M.splits : local;
+    const int tmi = tl / M.tiles_n, tn = tl % M.tiles_n;
     const int mt = (M.M + 63) / 64;
     const int b = tmi / mt, tm = tmi % mt;
     const Addr A = P.addrs[M.a_addr];
     const Addr B = P.addrs[M.b_addr];
+    const int kbeg = M.splits > 1 ? split * M.k_split : 0;
+    const int kend = M.splits > 1 ? min(M.K, kbeg + M.k_split) : M.K;
     float acc[2][8];
 #pragma unroll
     for (int i = 0; i < 2; ++i)
 #pragma unroll
       for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
-    for (int k0 = 0; k0 < M.K; k0 += 16) {
+    for (int k0 = kbeg; k0 < kend; k0 += 16) {
       __syncthreads();
       float av[4], bv[4];
 #pragma unroll
@@ -948,8 +953,8 @@ __device__ __noinline__ void run_gemm_simt(const Params& P, const Stage& st, cha
         int e = tid + q * kThreads;
         int kk = e >> 6, i = e & 63;
         int m = tm * 64 + i, n = tn * 64 + i, k = k0 + kk;
-        av[q] = (m < M.M && k < M.K) ? ld1(P, A, addr_off(P, A, (int64_t)b * M.M + m, k)) : 0.f;
-        bv[q] = (n < M.N && k < M.K) ? ld1(P, B, addr_off(P, B, (int64_t)b * M.N + n, k)) : 0.f;
+        av[q] = (m < M.M && k < kend) ? ld1(P, A, addr_off(P, A, (int64_t)b * M.M + m, k)) : 0.f;
+        bv[q] = (n < M.N && k < kend) ? ld1(P, B, addr_off(P, B, (int64_t)b * M.N + n, k)) : 0.f;
       }
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
@@ -973,6 +978,41 @@ __device__ __noinline__ void run_gemm_simt(const Params& P, const Stage& st, cha
           acc[0][j] = fmaf(a0, bvv, acc[0][j]);
           acc[1][j] = fmaf(a1, bvv, acc[1][j]);
         }
+      }
+    }
+    if (M.splits > 1) {
+      // partials into the fp32 tile accumulator (vector reductions into L2); the last split to arrive
+      // (per-tile counter) runs the fused chain on the sum and re-zeroes the tile
+      float* accbuf = (float*)P.ws_data + M.acc_off + (int64_t)tl * 64 * 64;
+#pragma unroll
+      for (int i = 0; i < 2; ++i) {
+        float* p = accbuf + (ty * 2 + i) * 64 + tx * 8;
+        asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(acc[i][0]), "f"(acc[i][1]),
+                     "f"(acc[i][2]), "f"(acc[i][3]) : "memory");
+        asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p + 4), "f"(acc[i][4]), "f"(acc[i][5]),
+                     "f"(acc[i][6]), "f"(acc[i][7]) : "memory");
+      }
+      __syncthreads();
+      SmemCtrl* ctl = ctrl_of(smem);
+      if (threadIdx.x == 0) {
+        unsigned* cnt = (unsigned*)P.ws_data + M.cnt_off + tl;
+        unsigned old;
+        asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(old) : "l"(cnt) : "memory");
+        ctl->flag = (old == (unsigned)(M.splits - 1)) ? 1 : 0;
+        if (ctl->flag) *cnt = 0u;   // self-cleaning for the next run
+      }
+      __syncthreads();
+      const bool last = ctl->flag != 0;
+      __syncthreads();   // the flag is read by every thread before the next task may rewrite it
+      if (!last) continue;
+#pragma unroll
+      for (int i = 0; i < 2; ++i) {
+        float4* p = reinterpret_cast<float4*>(accbuf + (ty * 2 + i) * 64 + tx * 8);
+        const float4 a0 = __ldcg(p), a1 = __ldcg(p + 1);
+        __stcg(p, make_float4(0.f, 0.f, 0.f, 0.f));
+        __stcg(p + 1, make_float4(0.f, 0.f, 0.f, 0.f));
+        acc[i][0] = a0.x; acc[i][1] = a0.y; acc[i][2] = a0.z; acc[i][3] = a0.w;
+        acc[i][4] = a1.x; acc[i][5] = a1.y; acc[i][6] = a1.z; acc[i][7] = a1.w;
       }
     }
 #pragma unroll

@@ -341,3 +341,62 @@ def se_module(cfg):
     y = g.ew("mul", x, gt)
     g.mark_output(y)
     return g, dict(x=x, W1=W1, b1=b1, W2=W2, b2=b2), x, y
+
+
+def mbconv(cfg):
+    """EfficientNet MBConv block as a TE program (same node order as oracle.graphs.mbconv): 1x1
+    convolutions as matmuls, the depthwise convolution as rolled, border-masked and weighted taps,
+    squeeze-and-excitation, BatchNorm as a per-channel affine; x [H*W, Cin] NHWC, batch 1."""
+    H, k, s, pad = cfg["hw"], cfg["k"], cfg["stride"], cfg["k"] // 2
+    cin, cout = cfg["cin"], cfg["cout"]
+    exp, S = cin * cfg["expand"], max(1, cin // 4)
+    Ho = H // s
+    g = L.Graph()
+    names = {}
+    x = g.placeholder((H * H, cin), L.F32, const=False)
+    a = x
+    if cfg["expand"] != 1:
+        names["We"] = g.placeholder((exp, cin))
+        a = g.matmul(x, names["We"], True, L.F32)
+        names["se"], names["be"] = g.placeholder((exp,)), g.placeholder((exp,))
+        a = g.ew("add", g.ew("mul", a, names["se"]), names["be"])
+        a = g.ew("mul", a, g.ew("sigmoid", a))
+    a3 = g.reshape(a, (H, H, exp))
+    acc = None
+    for i in range(k):
+        for j in range(k):
+            t = i * k + j
+            if i == pad and j == pad:
+                term = a3
+            else:
+                r = g.roll(a3, (pad - i, pad - j, 0))
+                names[f"m{t}"] = g.placeholder((H, H, 1))
+                term = g.ew("mul", r, names[f"m{t}"])
+            names[f"w{t}"] = g.placeholder((exp,))
+            term = g.ew("mul", term, names[f"w{t}"])
+            acc = term if acc is None else g.ew("add", acc, term)
+    if s != 1:
+        acc = g.slice(acc, (0, 0, 0), (H, H, exp), (s, s, 1))
+    d = g.reshape(acc, (Ho * Ho, exp))
+    names["sd"], names["bd"] = g.placeholder((exp,)), g.placeholder((exp,))
+    d = g.ew("add", g.ew("mul", d, names["sd"]), names["bd"])
+    d = g.ew("mul", d, g.ew("sigmoid", d))
+    p = g.reduce("mean", d, 0, True)
+    names["W1"] = g.placeholder((S, exp))
+    h = g.matmul(p, names["W1"], True, L.F32)
+    names["b1"] = g.placeholder((S,))
+    h = g.ew("add", h, names["b1"])
+    h = g.ew("mul", h, g.ew("sigmoid", h))
+    names["W2"] = g.placeholder((exp, S))
+    gt = g.matmul(h, names["W2"], True, L.F32)
+    names["b2"] = g.placeholder((exp,))
+    gt = g.ew("sigmoid", g.ew("add", gt, names["b2"]))
+    d = g.ew("mul", d, gt)
+    names["Wp"] = g.placeholder((cout, exp))
+    y = g.matmul(d, names["Wp"], True, L.F32)
+    names["sp"], names["bp"] = g.placeholder((cout,)), g.placeholder((cout,))
+    y = g.ew("add", g.ew("mul", y, names["sp"]), names["bp"])
+    if s == 1 and cin == cout:
+        y = g.ew("add", y, x)
+    g.mark_output(y)
+    return g, names, x, y

@@ -286,3 +286,64 @@ def se_params(cfg: dict) -> dict:
     C, S = cfg["channels"], cfg["squeeze"]
     return dict(W1=normal(701, (S, C), std=1.0 / np.sqrt(C)), b1=normal(702, (S,), std=0.02),
                 W2=normal(703, (C, S), std=1.0 / np.sqrt(S)), b2=normal(704, (C,), std=0.02))
+
+
+# ---------------------------------------------------------------- EfficientNet MBConv blocks M0-M9
+# The first efficientnet_b0 block (torchvision MBConvConfig) with each sub-module shape of SE_CONFIGS:
+# (input channels, output channels, expand ratio, depthwise kernel, stride, input height = width).
+MBCONV_CONFIGS = [
+    dict(name=f"M{i}", cin=ci, cout=co, expand=e, k=k, stride=s, hw=h)
+    for i, (ci, co, e, k, s, h) in enumerate([
+        (32, 16, 1, 3, 1, 112), (16, 24, 6, 3, 2, 112), (24, 24, 6, 3, 1, 56), (24, 40, 6, 5, 2, 56),
+        (40, 40, 6, 5, 1, 28), (40, 80, 6, 3, 2, 28), (80, 80, 6, 3, 1, 14), (112, 112, 6, 5, 1, 14),
+        (112, 192, 6, 5, 2, 14), (192, 192, 6, 5, 1, 7)])
+]
+
+
+def mbconv_dims(cfg: dict) -> dict:
+    """Derived sizes: expanded channels, squeeze width (torchvision: max(1, cin // 4)), output height."""
+    exp = cfg["cin"] * cfg["expand"]
+    return dict(exp=exp, squeeze=max(1, cfg["cin"] // 4), hw_out=cfg["hw"] // cfg["stride"], pad=cfg["k"] // 2)
+
+
+def mbconv_input(cfg: dict, seed: int = INPUT_SEED) -> np.ndarray:
+    """x [H*W, Cin] fp32 ~ N(0, 1) (NHWC, batch 1)."""
+    return normal(seed, (cfg["hw"] * cfg["hw"], cfg["cin"]))
+
+
+def mbconv_params(cfg: dict) -> dict:
+    """Random-init weights of one MBConv block, BatchNorm in inference form (per-channel scale s and
+    bias b: y = x * s + b).  1x1 convolutions as [out, in] matrices, the depthwise kernel as one [C]
+    vector per tap t = i * k + j; SE as in se_params.  fp32."""
+    d = mbconv_dims(cfg)
+    cin, cout, exp, S, k = cfg["cin"], cfg["cout"], d["exp"], d["squeeze"], cfg["k"]
+    base = 900 + 100 * cfg["k"] + cfg["cin"]
+    p = {}
+    if cfg["expand"] != 1:
+        p.update(We=normal(base + 1, (exp, cin), std=1.0 / np.sqrt(cin)), se=normal(base + 2, (exp,), std=0.1, mean=1.0),
+                 be=normal(base + 3, (exp,), std=0.1))
+    for t in range(k * k):
+        p[f"w{t}"] = normal(base + 10 + t, (exp,), std=1.0 / k)
+    p.update(sd=normal(base + 4, (exp,), std=0.1, mean=1.0), bd=normal(base + 5, (exp,), std=0.1),
+             W1=normal(base + 6, (S, exp), std=1.0 / np.sqrt(exp)), b1=normal(base + 7, (S,), std=0.02),
+             W2=normal(base + 8, (exp, S), std=1.0 / np.sqrt(S)), b2=normal(base + 9, (exp,), std=0.02),
+             Wp=normal(base + 40, (cout, exp), std=1.0 / np.sqrt(exp)), sp=normal(base + 41, (cout,), std=0.1, mean=1.0),
+             bp=normal(base + 42, (cout,), std=0.1))
+    return p
+
+
+def mbconv_masks(cfg: dict) -> dict:
+    """Zero-padding of the depthwise convolution as data: m{t}[h, w] = 1 iff input pixel (h + i - pad,
+    w + j - pad) of tap t = i * k + j lies inside the image (a structural constant, like the Swin
+    shifted-window mask).  [H, W, 1] fp32 per off-centre tap."""
+    H, k, pad = cfg["hw"], cfg["k"], cfg["k"] // 2
+    out = {}
+    h = np.arange(H)
+    for i in range(k):
+        for j in range(k):
+            if i == pad and j == pad:
+                continue
+            mh = ((h + i - pad) >= 0) & ((h + i - pad) < H)
+            mw = ((h + j - pad) >= 0) & ((h + j - pad) < H)
+            out[f"m{i * k + j}"] = (mh[:, None] & mw[None, :]).astype(np.float32).reshape(H, H, 1)
+    return out

@@ -1,5 +1,5 @@
 """Slowest stages of a model on the generic executor (CTA-0 stage marks).
-usage: python tools/profile_generic.py <bert|lstm|mmoe|swin> [flags]"""
+usage: python tools/profile_generic.py <bert|lstm|mmoe|swin|mbconv:IDX> [flags]"""
 import collections
 import os
 import sys
@@ -14,7 +14,17 @@ from paper_conf_asplos_xiazswwyfc24_b200.session import session  # noqa: E402
 
 name = sys.argv[1]
 flags = int(sys.argv[2]) if len(sys.argv) > 2 else L.FLAG_NO_PATTERN
-g, feed, outs = graph_and_feed(name)
+if name.startswith("mbconv:"):
+    import synth
+    from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+    cfg = synth.MBCONV_CONFIGS[int(name.split(":")[1])]
+    g, nm, gx, gy = M.mbconv(cfg)
+    feed = {nm[k]: v for k, v in {**synth.mbconv_params(cfg), **synth.mbconv_masks(cfg)}.items()}
+    feed[gx] = synth.mbconv_input(cfg)
+    outs = [gy]
+    flags = int(sys.argv[2]) if len(sys.argv) > 2 else 0
+else:
+    g, feed, outs = graph_and_feed(name)
 plan = g.partition(L.device_query(0), flags)
 plan.set_profiling(True)
 s = session(g, plan, feed, outs)
