@@ -498,6 +498,27 @@ def main():
                                     "modules": se_rows,
                                     "geomean_speedup_vs_unfused": float(np.exp(np.mean([np.log(r["speedup"]) for r in se_rows]))),
                                     "paper_a100": "Fig. 6: 1.31x global sync, 1.84x data reuse over unfused (avg)"}
+        # EfficientNet MBConv blocks M0-M9: the pattern kernel (one persistent launch, Fig. 5(c)) against
+        # the unfused one-kernel-per-TE path
+        progress("EfficientNet MBConv blocks")
+        mb_rows = []
+        for cfg in _synth.MBCONV_CONFIGS:
+            ps_ = {**_synth.mbconv_params(cfg), **_synth.mbconv_masks(cfg)}
+            g_, nm_, gx_, gy_ = M.mbconv(cfg)
+            row = {"module": cfg["name"], "cin": cfg["cin"], "cout": cfg["cout"], "k": cfg["k"], "stride": cfg["stride"],
+                   "hw": cfg["hw"]}
+            for key, fl in (("pattern_us", 0), ("unfused_us", L.FLAG_UNFUSED)):
+                pl_ = g_.partition(L.device_query(local), fl)
+                ss_ = _session(g_, pl_, {nm_[k]: v for k, v in ps_.items()} | {gx_: _synth.mbconv_input(cfg)}, [gy_],
+                               device=f"cuda:{local}")
+                row[key] = statistics.median(time_steps(ss_, 20, 3, flush, stream)) * 1e3
+                del ss_, pl_
+            row["speedup"] = row["unfused_us"] / row["pattern_us"]
+            mb_rows.append(row)
+        extra["efficientnet_mbconv"] = {"workload": "EfficientNet-b0 MBConv blocks M0-M9 (fp32, batch 1)",
+                                        "modules": mb_rows,
+                                        "geomean_speedup_vs_unfused": float(np.exp(np.mean([np.log(r["speedup"]) for r in mb_rows]))),
+                                        "kernel": "kernels/mbconv.cu (one persistent launch, Fig. 5(c))"}
         # Swin-B runs in a child process (fresh CUDA context) with a time limit: a launch that trips a
         # kernel watchdog must not take the whole bench line with it
         progress("Swin-B (child process)")

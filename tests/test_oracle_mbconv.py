@@ -80,3 +80,18 @@ def test_mbconv_library_graph_matches_oracle():
             op, shp, _ = g.node(i)
             assert op == opmap[nd["op"]] and shp == shapes[i], i
         assert g.partition(L.device_b200()).num_subprograms() >= 1
+
+
+def test_mbconv_pattern_matcher():
+    """Every module M0-M9 is recognised by the MBConv pattern lowering (one persistent launch); the
+    ablation flags keep the generic executor; a program that is not exactly the block is refused."""
+    from paper_conf_asplos_xiazswwyfc24_b200 import _lib as L
+    from paper_conf_asplos_xiazswwyfc24_b200 import models as M
+    for cfg in synth.MBCONV_CONFIGS:
+        g = M.mbconv(cfg)[0]
+        d = g.partition(L.device_b200()).describe()
+        assert "pattern mbconv: " in d and "pattern mbconv: not used" not in d, cfg["name"]
+        assert g.partition(L.device_b200()).exec_info()["launches"] == 1
+        assert "pattern mbconv: not used" in g.partition(L.device_b200(), L.FLAG_NO_PATTERN).describe()
+    g = M.se_module(synth.SE_CONFIGS[0])[0]
+    assert "pattern mbconv: not used" in g.partition(L.device_b200()).describe()
