@@ -490,10 +490,10 @@ souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t
       if (barriers) *barriers = 3;
       return;
     }
-    if (P.mb.on) {   // expand, depthwise + pool, pooled, fc1, fc2 + project (+ split-K finish)
+    if (P.mb.on) {   // expand | depthwise + pool | fc1 | gates + project (+ split-K finish)
       if (launches) *launches = 1;
-      if (stages) *stages = 5;
-      if (barriers) *barriers = 4;
+      if (stages) *stages = 4;
+      if (barriers) *barriers = 3;
       return;
     }
     if (P.swin.on) {   // one kernel per fused subprogram, replayed as one CUDA graph

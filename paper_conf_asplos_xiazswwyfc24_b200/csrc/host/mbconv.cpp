@@ -1,6 +1,7 @@
 // EfficientNet MBConv pattern (Fig. 5 / 6): strict TE match of the block's program, workspace
 // layout and launch of kernels/mbconv.cu.
 #include <cmath>
+#include <cstdlib>
 #include <sstream>
 #include <string>
 
@@ -192,11 +193,11 @@ souffle_status mbconv_run(Plan& p, void* ws, void* stream) {
   prm.y = (float*)p.buf_ptr[p.node_buf[mp.y]];
   prm.a = (float*)(base + mp.o_a);
   prm.d = (float*)(base + mp.o_d);
-  prm.part = (float*)(base + mp.o_part);
   prm.pooled = (float*)(base + mp.o_pooled);
   prm.h = (float*)(base + mp.o_h);
   prm.acc = (float*)(base + mp.o_acc);
   prm.ctrl = (unsigned*)(base + mp.o_ctrl);
+  if (std::getenv("SOUFFLE_MB_PROF")) prm.prof = (unsigned long long*)(base + mp.o_ctrl + 64);   // 8 stamps
   prm.H = mp.H; prm.cin = mp.cin; prm.E = mp.E; prm.k = mp.k; prm.stride = mp.stride; prm.S = mp.S;
   prm.cout = mp.cout; prm.residual = mp.residual;
   cudaError_t e = mbconv_launch(prm, mp.grid, (cudaStream_t)stream);

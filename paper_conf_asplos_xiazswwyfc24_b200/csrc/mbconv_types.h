@@ -36,11 +36,11 @@ struct MbParams {
   float* y;                       // [Ho*Ho][cout]
   float* a;                       // workspace [H*H][E] (expand output)
   float* d;                       // workspace [Ho*Ho][E] (depthwise output)
-  float* part;                    // workspace [grid][E] per-CTA pool partial sums
-  float* pooled;                  // [E]
+  float* pooled;                  // [E] channel sums of d (zero between launches)
   float* h;                       // [S]
   float* acc;                     // [Ho*Ho][cout] split-K accumulator of the project GEMM
-  unsigned* ctrl;                 // [0..4] grid barriers, [5] exit counter
+  unsigned* ctrl;                 // [0..3] grid barriers, [5] exit counter
+  unsigned long long* prof;       // debug (SOUFFLE_MB_PROF): %globaltimer of CTA 0 at the phase boundaries [8]
   int32_t H, cin, E, k, stride, S, cout, residual;
 };
 
