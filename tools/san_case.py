@@ -1,5 +1,5 @@
 """One small launch of a kernel family, checked against the oracle (for compute-sanitizer runs).
-usage: python tools/san_case.py bert_small | swin_small | generic_tiny | rowwise | swin_generic
+usage: python tools/san_case.py bert_small | swin_small | generic_tiny | rowwise | swin_generic | mbconv:IDX
 (rowwise / swin_generic / generic_tiny exercise the generic executor's row-block stages and tensor cache;
 SOUFFLE_CACHE_FLOATS=2048 forces LRU spills)"""
 import os
@@ -25,6 +25,18 @@ if which in ("bert_small", "generic_tiny"):
     g, gX, gpl, gy = M.bert(cfg)
     plan = g.partition(L.device_query(0))
     s = session(g, plan, og.bert_feed(gX, gpl, x, w), [gy])
+    s.run()
+    out = s.result(gy)
+elif which.startswith("mbconv:"):
+    cfg = synth.MBCONV_CONFIGS[int(which.split(":")[1])]
+    p = {**synth.mbconv_params(cfg), **synth.mbconv_masks(cfg)}
+    spec, on, ox, oy = og.mbconv(cfg)
+    x = synth.mbconv_input(cfg)
+    ref = te.evaluate(spec, {on[k]: v for k, v in p.items()} | {ox: x})[oy]
+    g, gn, gx, gy = M.mbconv(cfg)
+    plan = g.partition(L.device_query(0))
+    s = session(g, plan, {gn[k]: v for k, v in p.items()} | {gx: x}, [gy])
+    s.run()
     s.run()
     out = s.result(gy)
 elif which == "rowwise":
