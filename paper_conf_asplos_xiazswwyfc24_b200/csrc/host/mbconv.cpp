@@ -14,6 +14,7 @@ namespace souffle {
 
 souffle_status fail(souffle_status c, const std::string& m);
 cudaError_t mbconv_launch(const MbParams& prm, int grid, cudaStream_t s);
+size_t mbconv_reuse_smem(int pix_blk, int E, int cout);
 
 namespace {
 int64_t al(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
@@ -65,7 +66,7 @@ void mbconv_match(const Graph& g, const Analysis& an, const souffle_device_desc&
   mp = MbPlan();
   for (int t = 0; t < MB_MAX_TAPS; ++t) mp.w[t] = mp.m[t] = -1;
   auto no = [&](const char* why) { mp.on = false; mp.why_not = why; };
-  if (flags != 0) return no("ablation flags select the generic executor");
+  if (flags != 0 && flags != SOUFFLE_FLAG_NO_PREFETCH) return no("ablation flags select the generic executor");
   const auto& N = g.nodes;
   if (N.size() < 40 || N[0].op != SOUFFLE_OP_PLACEHOLDER || N[0].shape.size() != 2 || N[0].is_const ||
       N[0].dtype != SOUFFLE_F32)
@@ -153,6 +154,12 @@ void mbconv_match(const Graph& g, const Analysis& an, const souffle_device_desc&
   mp.y = y;
   mp.H = (int)H; mp.cin = (int)cin; mp.E = (int)E; mp.k = (int)k; mp.stride = (int)stride; mp.S = (int)S;
   mp.cout = (int)cout; mp.grid = sms; mp.num_sp = an.num_sp;
+  // data reuse (Fig. 5(d)): the CTA's d block and the whole Wp in shared memory, when Wp is small and
+  // each CTA owns enough pixels for the saved d round trip to outweigh staging Wp (measured: it pays
+  // at 85 pixels per CTA, is neutral at 22 and costs at 6, profiles/r02_mbconv_ablation.jsonl)
+  mp.pix_blk = (int)((Ho * Ho + sms - 1) / sms);
+  mp.reuse = flags == 0 && mp.pix_blk >= 16 && (size_t)cout * E * 4 <= 64 * 1024 &&
+             mbconv_reuse_smem(mp.pix_blk, (int)E, (int)cout) <= (size_t)MB_MAX_REUSE_SMEM;
   int64_t o = 0;
   mp.o_ctrl = o; o = al(o + 256, 256);
   mp.o_a = o; o = al(o + 4 * (mp.We >= 0 ? HW * E : 0), 256);
@@ -173,7 +180,8 @@ std::string mbconv_describe(const MbPlan& mp) {
   }
   os << "pattern mbconv: " << mp.cin << " -> " << mp.cout << " channels, expand " << mp.E / mp.cin << ", depthwise "
      << mp.k << "x" << mp.k << " stride " << mp.stride << ", " << mp.H << "x" << mp.H << ", SE " << mp.S
-     << (mp.residual ? ", residual" : "") << " -> 1 persistent launch (kernels/mbconv.cu), " << mp.grid
+     << (mp.residual ? ", residual" : "") << " -> 1 persistent launch (kernels/mbconv.cu), "
+     << (mp.reuse ? "d reused from shared memory (Fig. 5(d)), " : "d through L2 (Fig. 5(c)), ") << mp.grid
      << " CTAs, 4-5 grid barriers (the partition's " << mp.num_sp << " subprogram(s) end at barriers of the launch)\n";
   return os.str();
 }
@@ -199,7 +207,7 @@ souffle_status mbconv_run(Plan& p, void* ws, void* stream) {
   prm.ctrl = (unsigned*)(base + mp.o_ctrl);
   if (std::getenv("SOUFFLE_MB_PROF")) prm.prof = (unsigned long long*)(base + mp.o_ctrl + 64);   // 8 stamps
   prm.H = mp.H; prm.cin = mp.cin; prm.E = mp.E; prm.k = mp.k; prm.stride = mp.stride; prm.S = mp.S;
-  prm.cout = mp.cout; prm.residual = mp.residual;
+  prm.cout = mp.cout; prm.residual = mp.residual; prm.reuse = mp.reuse; prm.pix_blk = mp.pix_blk;
   cudaError_t e = mbconv_launch(prm, mp.grid, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("mbconv launch: ") + cudaGetErrorString(e));
   return SOUFFLE_OK;

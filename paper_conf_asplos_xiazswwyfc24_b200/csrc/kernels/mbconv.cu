@@ -128,6 +128,9 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
   __shared__ float tsm[2 * 16 * 65];   // GEMM operand slabs
   __shared__ float pool[MB_MAX_E];
   __shared__ float g[MB_MAX_E];
+  extern __shared__ float dyn[];       // data reuse: [pix_blk][E] depthwise output, then [cout][E + 1] Wp
+  float* d_s = dyn;
+  float* wp_s = dyn + P.pix_blk * P.E;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int H = P.H, E = P.E, k = P.k, s = P.stride, pad = k / 2;
   const int HW = H * H, Ho = H / s, HWo = Ho * Ho;
@@ -145,7 +148,7 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
   // the project GEMM splits K over the idle CTAs when it has few output tiles (the narrow late modules:
   // 49 pixels x 1152 channels); its fp32 accumulator is cleared here, long before phase 4
   const int ptm = (HWo + 31) / 32, ptn = (P.cout + 31) / 32, ptiles = ptm * ptn;
-  const int psplit = 2 * ptiles <= (int)gridDim.x ? min((int)gridDim.x / ptiles, (E + 31) / 32) : 1;
+  const int psplit = !P.reuse && 2 * ptiles <= (int)gridDim.x ? min((int)gridDim.x / ptiles, (E + 31) / 32) : 1;
   if (psplit > 1)
     for (int i = blockIdx.x * MB_THREADS + tid; i < HWo * P.cout; i += gridDim.x * MB_THREADS) P.acc[i] = 0.f;
   // ---- 2: depthwise convolution (+ BN + SiLU) of this CTA's block of output pixels; (pixel, channel)
@@ -155,8 +158,9 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
   {
     // the (pixel, channel) pairs of the whole output split evenly over the grid (a few wide pixels,
     // e.g. 7 x 7 x 1152, still keep every CTA busy)
+    // (data reuse: whole pixel blocks, so that this CTA's d block stays in its shared memory)
     const int64_t total = (int64_t)HWo * E;
-    const int64_t per = (total + gridDim.x - 1) / gridDim.x;
+    const int64_t per = P.reuse ? (int64_t)P.pix_blk * E : (total + gridDim.x - 1) / gridDim.x;
     const int64_t i0 = blockIdx.x * per, i1 = min(total, i0 + per);
     for (int e = tid; e < E; e += MB_THREADS) pool[e] = 0.f;
     __syncthreads();
@@ -180,7 +184,8 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
         }
       }
       const float dv = silu(acc * __ldg(P.sd + e) + __ldg(P.bd + e));
-      P.d[(int64_t)q * E + e] = dv;
+      if (P.reuse) d_s[idx - i0] = dv;
+      else P.d[(int64_t)q * E + e] = dv;
       atomicAdd(&pool[e], dv);
     }
     __syncthreads();
@@ -217,6 +222,28 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
     __syncthreads();
   };
   // ---- 4: project convolution on the rescaled d (+ BN, + residual)
+  if (P.reuse) {
+    // ---- 4 (data reuse, Fig. 5(d)): this CTA's own pixels, d from shared memory, Wp staged beside it
+    const int q0 = blockIdx.x * P.pix_blk, nq = min(P.pix_blk, HWo - q0);
+    if (nq > 0) {
+      gates(0, E);
+      for (int i = tid; i < P.cout * E; i += MB_THREADS) wp_s[(i / E) * (E + 1) + i % E] = __ldg(P.Wp + i);
+      for (int i = tid; i < nq * E; i += MB_THREADS) d_s[i] *= g[i % E];
+      __syncthreads();
+      for (int o = tid; o < nq * P.cout; o += MB_THREADS) {
+        const int qq = o / P.cout, n = o % P.cout;
+        const float* dr = d_s + qq * E;
+        const float* wr = wp_s + n * (E + 1);   // padded rows: consecutive n on distinct banks
+        float acc = 0.f;
+#pragma unroll 4
+        for (int e = 0; e < E; ++e) acc = fmaf(dr[e], wr[e], acc);
+        const int m = q0 + qq;
+        float y = acc * __ldg(P.sp + n) + __ldg(P.bp + n);
+        if (P.residual) y += __ldg(P.x + (int64_t)m * P.cout + n);
+        P.y[(int64_t)m * P.cout + n] = y;
+      }
+    }
+  } else {
   auto finish = [&](int m, int n, float v) {
     float y = v * __ldg(P.sp + n) + __ldg(P.bp + n);
     if (P.residual) y += __ldg(P.x + (int64_t)m * P.cout + n);
@@ -240,6 +267,7 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
     for (int i = blockIdx.x * MB_THREADS + tid; i < HWo * P.cout; i += gridDim.x * MB_THREADS)
       finish(i / P.cout, i % P.cout, __ldcg(P.acc + i));
   }
+  }
   stamp(P, 6);
   // ---- exit: the last CTA resets the barrier counters and the pooled sums for the next launch
   __syncthreads();
@@ -259,11 +287,13 @@ __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_cons
 
 }  // namespace mb
 
+size_t mbconv_reuse_smem(int pix_blk, int E, int cout) { return 4 * ((size_t)pix_blk * E + (size_t)cout * (E + 1)); }
+
 cudaError_t mbconv_launch(const MbParams& prm, int grid, cudaStream_t s) {
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(MB_THREADS);
-  cfg.dynamicSmemBytes = 0;
+  cfg.dynamicSmemBytes = prm.reuse ? mbconv_reuse_smem(prm.pix_blk, prm.E, prm.cout) : 0;
   cfg.stream = s;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeCooperative;   // the grid barriers need every CTA co-resident
@@ -271,6 +301,10 @@ cudaError_t mbconv_launch(const MbParams& prm, int grid, cudaStream_t s) {
   cfg.attrs = at;
   cfg.numAttrs = 1;
   void (*fn)(MbParams) = prm.k == 3 ? mb::mbconv_kernel<3> : prm.k == 5 ? mb::mbconv_kernel<5> : mb::mbconv_kernel<0>;
+  if (prm.reuse) {
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, MB_MAX_REUSE_SMEM);
+    if (e != cudaSuccess) return e;
+  }
   return cudaLaunchKernelEx(&cfg, fn, prm);
 }
 

@@ -15,7 +15,8 @@
 
 namespace souffle {
 
-enum { MB_THREADS = 256, MB_MAX_KS = 5, MB_MAX_TAPS = MB_MAX_KS * MB_MAX_KS, MB_MAX_E = 2048 };
+enum { MB_THREADS = 256, MB_MAX_KS = 5, MB_MAX_TAPS = MB_MAX_KS * MB_MAX_KS, MB_MAX_E = 2048,
+       MB_MAX_REUSE_SMEM = 160 * 1024 };
 
 struct MbParams {
   const float* x;                 // [H*H][cin]
@@ -42,6 +43,8 @@ struct MbParams {
   unsigned* ctrl;                 // [0..3] grid barriers, [5] exit counter
   unsigned long long* prof;       // debug (SOUFFLE_MB_PROF): %globaltimer of CTA 0 at the phase boundaries [8]
   int32_t H, cin, E, k, stride, S, cout, residual;
+  int32_t reuse;     // 1: Fig. 5(d) data reuse (d block + Wp in shared memory), 0: d through L2
+  int32_t pix_blk;   // reuse: output pixels per CTA
 };
 
 }  // namespace souffle

@@ -34,17 +34,22 @@ def _case(cfg):
     return g, {gnames[k]: v for k, v in p.items()} | {gx: x}, gy, ref
 
 
+@pytest.mark.parametrize("flags", [0, L.FLAG_NO_PREFETCH], ids=["reuse", "global_sync"])
 @pytest.mark.parametrize("cfg", synth.MBCONV_CONFIGS, ids=[c["name"] for c in synth.MBCONV_CONFIGS])
-def test_mbconv_pattern(cfg, record_err):
+def test_mbconv_pattern(cfg, flags, record_err):
+    """The pattern kernel: Fig. 5(d) (d kept in shared memory where the planner chooses it) and
+    Fig. 5(c) (NO_PREFETCH: d through L2)."""
     g, feed, gy, ref = _case(cfg)
-    plan = g.partition(L.device_query(0))
+    plan = g.partition(L.device_query(0), flags)
+    if flags:
+        assert "Fig. 5(c)" in plan.describe()
     assert "pattern mbconv: " in plan.describe() and "not used" not in plan.describe().split("pattern mbconv")[1][:20]
     s = session(g, plan, feed, [gy])
     s.run()
     out = s.result(gy)
     s.run()                                   # a second launch reuses the workspace (barrier counters reset)
-    record_err(rel_err(out, ref), 1e-4, module=cfg["name"], variant="pattern")
-    record_err(rel_err(s.result(gy), ref), 1e-4, module=cfg["name"], variant="pattern_again")
+    record_err(rel_err(out, ref), 1e-4, module=cfg["name"], variant=f"pattern_{flags}")
+    record_err(rel_err(s.result(gy), ref), 1e-4, module=cfg["name"], variant=f"pattern_{flags}_again")
 
 
 @pytest.mark.parametrize("cfg", synth.MBCONV_CONFIGS, ids=[c["name"] for c in synth.MBCONV_CONFIGS])

@@ -2,7 +2,8 @@
 pins the TE program to torchvision): M0-M9 in (a) unfused: one launch per TE; (b) fused: the generic
 executor's fused stages launched one by one (NO_GLOBAL_SYNC); the generic executor with one launch per
 subprogram, without and with §6.5 reuse; (c) global sync: the MBConv pattern kernel, one persistent
-launch (kernels/mbconv.cu).
+launch (kernels/mbconv.cu, NO_PREFETCH: d through L2); (d) data reuse: the same kernel with each CTA's
+d block kept in shared memory (where the planner chooses it).
 Median of 30 L2-flushed runs; one JSON object per module.  usage: python tools/ablation_mbconv.py [out.jsonl]"""
 import json
 import os
@@ -20,7 +21,7 @@ from paper_conf_asplos_xiazswwyfc24_b200.session import session  # noqa: E402
 
 VERSIONS = [("unfused", L.FLAG_UNFUSED), ("fused", L.FLAG_NO_GLOBAL_SYNC),
             ("generic_global_sync", L.FLAG_NO_PATTERN | L.FLAG_NO_PREFETCH), ("generic_reuse", L.FLAG_NO_PATTERN),
-            ("global_sync", 0)]
+            ("global_sync", L.FLAG_NO_PREFETCH), ("data_reuse", 0)]
 
 
 def run(out_path=None):
@@ -40,7 +41,7 @@ def run(out_path=None):
             row[name + "_launches"] = info["launches"]
             row[name + "_barriers"] = info["barriers"]
             del s, plan
-        for name in ("fused", "generic_global_sync", "generic_reuse", "global_sync"):
+        for name in ("fused", "generic_global_sync", "generic_reuse", "global_sync", "data_reuse"):
             row["speedup_" + name + "_vs_unfused"] = row["unfused_us"] / row[name + "_us"]
         rows.append(row)
         print(json.dumps(row), flush=True)
