@@ -3,7 +3,9 @@
 // Table 5 (one kernel).
 #include <cstdlib>
 #include <cstring>
+#include <array>
 #include <sstream>
+#include <vector>
 #include <string>
 
 #include <cuda_runtime.h>
@@ -151,8 +153,60 @@ std::string mmoe_describe(const MmoePlan& mp) {
   return os.str();
 }
 
+// parameter staging table (kernels/mmoe.cu): the shared-memory layout of the kernel, the bound
+// pointers and the unit prefix sums, uploaded once per workspace initialisation
+souffle_status mmoe_init(Plan& p, void* ws, void* stream) {
+  const MmoePlan& mp = p.mmoe;
+  auto ptr = [&](int node) -> uint64_t { return (uint64_t)(uintptr_t)p.buf_ptr[p.node_buf[node]]; };
+  const int64_t es = mp.w_f32 ? 4 : 2, B = mp.B, D = mp.D, E = mp.E, De = mp.De, T = mp.T, Th = mp.Th;
+  const int64_t R = E * De + T * E;
+  auto a16 = [](int64_t x) { return (x + 15) & ~int64_t(15); };
+  const int64_t oW1 = 0, oWt = a16(R * D * es), oWo = oWt + a16(T * Th * De * es), oxs = oWo + a16(T * Th * es);
+  const int64_t ob1 = oxs + 4 * B * D, obt = ob1 + 4 * R, obo = obt + 4 * T * Th;
+  std::vector<uint32_t> tab(2 * MMOE_SEG * 4, 0u);
+  int nseg[2] = {0, 0};
+  for (int t = 0; t < 2; ++t) {
+    std::vector<std::array<int64_t, 3>> segs;   // (src, smem offset, units)
+    if (t == 0) {
+      for (int e = 0; e < E; ++e) segs.push_back({(int64_t)ptr(mp.We[e]), oW1 + e * De * D * es, De * D * es / 16});
+      for (int k = 0; k < T; ++k) {
+        segs.push_back({(int64_t)ptr(mp.Wg[k]), oW1 + (E * De + k * E) * D * es, E * D * es / 16});
+        segs.push_back({(int64_t)ptr(mp.Wt[k]), oWt + k * Th * De * es, Th * De * es / 16});
+        segs.push_back({(int64_t)ptr(mp.Wo[k]), oWo + k * Th * es, Th * es / 16});
+      }
+    } else {
+      segs.push_back({(int64_t)ptr(mp.x), oxs, B * D});
+      for (int e = 0; e < E; ++e) segs.push_back({(int64_t)ptr(mp.be[e]), ob1 + 4 * e * De, De});
+      for (int k = 0; k < T; ++k) {
+        segs.push_back({(int64_t)ptr(mp.bg[k]), ob1 + 4 * (E * De + k * E), E});
+        segs.push_back({(int64_t)ptr(mp.bt[k]), obt + 4 * k * Th, Th});
+        segs.push_back({(int64_t)ptr(mp.bo[k]), obo + 4 * k, 1});
+      }
+    }
+    if ((int)segs.size() + 1 > MMOE_SEG) return fail(SOUFFLE_E_UNSUPPORTED, "MMoE staging table overflow");
+    int64_t pre = 0;
+    for (size_t j = 0; j <= segs.size(); ++j) {
+      uint32_t* e = &tab[(t * MMOE_SEG + j) * 4];
+      const uint64_t src = j < segs.size() ? (uint64_t)segs[j][0] : 0;
+      e[0] = (uint32_t)src;
+      e[1] = (uint32_t)(src >> 32);
+      e[2] = j < segs.size() ? (uint32_t)segs[j][1] : 0u;
+      e[3] = (uint32_t)pre;
+      if (j < segs.size()) pre += segs[j][2];
+    }
+    nseg[t] = (int)segs.size();
+  }
+  p.mmoe.nseg[0] = nseg[0];
+  p.mmoe.nseg[1] = nseg[1];
+  cudaError_t e = cudaMemcpyAsync(ws, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice, (cudaStream_t)stream);
+  if (e == cudaSuccess) e = cudaStreamSynchronize((cudaStream_t)stream);   // the host table is a local
+  if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("mmoe workspace init: ") + cudaGetErrorString(e));
+  p.inited_ws = ws;
+  p.dirty = false;
+  return SOUFFLE_OK;
+}
+
 souffle_status mmoe_run(Plan& p, void* ws, void* stream) {
-  (void)ws;
   MmoePlan& mp = p.mmoe;
   auto ptr = [&](int node) -> void* { return p.buf_ptr[p.node_buf[node]]; };
   MmoeParams prm;
@@ -174,6 +228,9 @@ souffle_status mmoe_run(Plan& p, void* ws, void* stream) {
   prm.B = mp.B; prm.D = mp.D; prm.E = mp.E; prm.De = mp.De; prm.T = mp.T; prm.Th = mp.Th;
   prm.w_f32 = mp.w_f32;
   prm.pad = std::getenv("SOUFFLE_MMOE_DEBUG") ? 1 : 0;   // debug: per-phase clock deltas (printf)
+  prm.seg = (const uint4*)ws;
+  prm.nseg[0] = mp.nseg[0];
+  prm.nseg[1] = mp.nseg[1];
   for (int k = 0; k < mp.E; ++k)
     if ((uintptr_t)prm.We[k] & 15) return fail(SOUFFLE_E_INVALID_ARG, "MMoE weights must be 16-byte aligned");
   for (int k = 0; k < mp.T; ++k)

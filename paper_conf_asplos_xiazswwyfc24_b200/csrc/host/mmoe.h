@@ -16,6 +16,7 @@ struct MmoePlan {
   int B = 0, D = 0, E = 0, De = 0, T = 0, Th = 0, w_f32 = 0;
   int x = -1;
   std::vector<int> We, be, Wg, bg, Wt, bt, Wo, bo, y;
+  int nseg[2] = {0, 0};   // staging-table segments (set at workspace initialisation)
 };
 
 void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp);

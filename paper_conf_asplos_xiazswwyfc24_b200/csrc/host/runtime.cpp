@@ -8,6 +8,7 @@
 #include <stdexcept>
 #include <string>
 
+#include "../mmoe_types.h"
 #include "plan.h"
 
 namespace souffle {
@@ -30,11 +31,12 @@ souffle_status swin_init(Plan& p, void* ws, void* stream);
 souffle_status swin_run(Plan& p, void* ws, void* stream);
 souffle_status se_run(Plan& p, void* ws, void* stream);
 souffle_status mbconv_run(Plan& p, void* ws, void* stream);
+souffle_status mmoe_init(Plan& p, void* ws, void* stream);
 
 size_t workspace_bytes(Plan& p) {
   if (p.bert.on) return (size_t)p.bert.total;
   if (p.lstm.on) return (size_t)p.lstm.total;
-  if (p.mmoe.on) return 256;
+  if (p.mmoe.on) return 2 * MMOE_SEG * 16;   // the parameter staging table
   if (p.swin.on) return (size_t)p.swin.total;
   if (p.se.on) return (size_t)p.se.total;
   if (p.mb.on) return (size_t)p.mb.total;
@@ -118,11 +120,7 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
     p.dirty = false;
     return SOUFFLE_OK;
   }
-  if (p.mmoe.on) {
-    p.inited_ws = ws;
-    p.dirty = false;
-    return SOUFFLE_OK;
-  }
+  if (p.mmoe.on) return mmoe_init(p, ws, stream);
   workspace_bytes(p);
   const WsLayout& w = p.ws;
   char* base = (char*)ws;

@@ -60,71 +60,37 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   // -- 16-byte weight segments and 4-byte vector segments -- then every thread loads its (up to 4 +
   // 1) elements of the concatenation before storing any (14 serial bulk-copy issues measured ~7 us,
   // per-segment load/store loops ~11 us).
-  constexpr int kSeg = MMOE_MAX_E + 3 * MMOE_MAX_T + 1;
+  constexpr int kSeg = MMOE_SEG;
   __shared__ const char* s_src[2][kSeg];
   __shared__ char* s_dst[2][kSeg];
-  __shared__ int s_pre[2][kSeg + 1];
+  __shared__ int s_pre[2][kSeg];
   __shared__ int s_nseg[2];
-  if (warp == 0) {
-    // segment table, one segment per lane (weights: We[0..E) then per task Wg, Wt, Wo; vectors: x,
-    // be[0..E) then per task bg, bt, bo), lengths prefix-summed with a warp scan
-    const int nw = E + 3 * T, nv = 1 + E + 3 * T;
-    for (int t = 0; t < 2; ++t) {
-      const int n = t == 0 ? nw : nv;
-      const char* src = nullptr;
-      char* dst = nullptr;
-      int units = 0;
-      if (lane < n) {
-        if (t == 0) {
-          if (lane < E) {
-            src = (const char*)P.We[lane]; dst = W1 + (int64_t)lane * De * D * es; units = De * D * es / 16;
-          } else {
-            const int k = (lane - E) / 3, which = (lane - E) % 3;
-            if (which == 0) { src = (const char*)P.Wg[k]; dst = W1 + (int64_t)(E * De + k * E) * D * es; units = E * D * es / 16; }
-            else if (which == 1) { src = (const char*)P.Wt[k]; dst = Wt + (int64_t)k * Th * De * es; units = Th * De * es / 16; }
-            else { src = (const char*)P.Wo[k]; dst = Wo + (int64_t)k * Th * es; units = Th * es / 16; }
-          }
-        } else {
-          if (lane == 0) { src = (const char*)P.x; dst = (char*)xs; units = B * D; }
-          else if (lane <= E) { src = (const char*)P.be[lane - 1]; dst = (char*)(b1 + (lane - 1) * De); units = De; }
-          else {
-            const int k = (lane - 1 - E) / 3, which = (lane - 1 - E) % 3;
-            if (which == 0) { src = (const char*)P.bg[k]; dst = (char*)(b1 + E * De + k * E); units = E; }
-            else if (which == 1) { src = (const char*)P.bt[k]; dst = (char*)(bt + k * Th); units = Th; }
-            else { src = (const char*)P.bo[k]; dst = (char*)(bo + k); units = 1; }
-          }
-        }
-      }
-      int incl = units;   // inclusive scan over the lanes
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += y;
-      }
-      if (lane < n) {
-        s_src[t][lane] = src;
-        s_dst[t][lane] = dst;
-        s_pre[t][lane] = incl - units;
-      }
-      if (lane == n - 1) {
-        s_pre[t][n] = incl;
-        s_nseg[t] = n;
-      }
+  // the segment table (weights: We[0..E) then per task Wg, Wt, Wo; vectors: x, be[0..E) then per task
+  // bg, bt, bo) was laid out on the host at workspace initialisation: one coalesced load per entry
+  if (tid < 2 * kSeg) {
+    const int t = tid / kSeg, j = tid % kSeg;
+    if (j <= P.nseg[t]) {
+      const uint4 e = __ldg(P.seg + tid);
+      s_src[t][j] = reinterpret_cast<const char*>(((unsigned long long)e.y << 32) | e.x);
+      s_dst[t][j] = smraw + e.z;
+      s_pre[t][j] = (int)e.w;
     }
+    if (j == 0) s_nseg[t] = P.nseg[t];
   }
   __syncthreads();
+  if (dbg && tid == 0) tk[2] = clock64();   // segment table built
   {
     constexpr int kW = 4;   // 16-byte units per thread (the MMoE parameters are <= 4 x 1024 x 16 B)
     uint4 wv[kW];
     int ws[kW], wo[kW];
     float fv;
     int fs = -1, fo = 0;
+    int sg = 0;   // segment of the previous unit: the units of a thread ascend, so the scan resumes
 #pragma unroll
     for (int j = 0; j < kW; ++j) {
       const int idx = tid + j * MMOE_THREADS;
       ws[j] = -1;
       if (idx < s_pre[0][s_nseg[0]]) {
-        int sg = 0;
         while (s_pre[0][sg + 1] <= idx) ++sg;
         ws[j] = sg;
         wo[j] = idx - s_pre[0][sg];
@@ -145,7 +111,6 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   }
   __syncthreads();
   if (dbg && tid == 0) tk[1] = clock64();
-  if (dbg && tid == 0) tk[2] = clock64();
   // ---- 1: fused expert + gate GEMM, 4 threads per (row, batch) output, k interleaved by 4 (the 8
   // outputs of a warp hit 32 distinct banks: row stride D = 100 floats = 4 banks), 2 shuffles
   for (int base = warp * 32; base < 4 * R * B; base += MMOE_THREADS) {   // warp-uniform trip count
@@ -155,6 +120,7 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
     const float* xr = xs + b * D;
     float s = 0.f;
     if (valid)
+#pragma unroll 8
       for (int k = part; k < D; k += 4) s = fmaf(xr[k], wsm(W1, r * D + k, f32), s);
     s += __shfl_xor_sync(0xffffffffu, s, 1);
     s += __shfl_xor_sync(0xffffffffu, s, 2);
@@ -185,6 +151,7 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
     const int b = i / (T * De), k = (i / De) % T, j = i % De;
     const float* g = o1 + b * R + E * De + k * E;
     float acc = g[0] * o1[b * R + j];
+#pragma unroll 4
     for (int e = 1; e < E; ++e) acc = acc + g[e] * o1[b * R + e * De + j];
     f[i] = acc;
   }
@@ -197,6 +164,7 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
     const int b = i / (T * Th), k = (i / Th) % T, r = i % Th;
     float s = 0.f;
     if (valid)
+#pragma unroll 4
       for (int j = part; j < De; j += 8) s = fmaf(f[(b * T + k) * De + j], wsm(Wt, (k * Th + r) * De + j, f32), s);
     s += __shfl_xor_sync(0xffffffffu, s, 4);
     s += __shfl_xor_sync(0xffffffffu, s, 2);
@@ -215,8 +183,8 @@ __global__ void __launch_bounds__(MMOE_THREADS, 1) mmoe_kernel(const __grid_cons
   }
   if (dbg && tid == 0) {
     tk[5] = clock64();
-    printf("mmoe clocks: params+issue %lld | bulk wait %lld | gemm %lld | softmax+mix %lld | towers %lld\n",
-           tk[1] - tk[0], tk[2] - tk[1], tk[3] - tk[2], tk[4] - tk[3], tk[5] - tk[4]);
+    printf("mmoe clocks: segment table %lld | parameter loads %lld | gemm %lld | softmax+mix %lld | towers %lld\n",
+           tk[2] - tk[0], tk[1] - tk[2], tk[3] - tk[1], tk[4] - tk[3], tk[5] - tk[4]);
   }
 }
 

@@ -3,10 +3,11 @@
 // expert GEMMs and the 2 gate GEMMs share x and run as one fused GEMM), Table 5 (one kernel).
 #pragma once
 #include <stdint.h>
+#include <vector_types.h>
 
 namespace souffle {
 
-enum { MMOE_THREADS = 1024, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
+enum { MMOE_SEG = 40, MMOE_THREADS = 1024, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
 
 struct MmoeParams {
   const float* x;                  // [B][D]
@@ -21,6 +22,11 @@ struct MmoeParams {
   float* y[MMOE_MAX_T];            // outputs [B][1]
   int32_t B, D, E, De, T, Th;
   int32_t w_f32, pad;
+  // parameter staging table, built on the host at workspace initialisation (pointers are known then;
+  // a re-bind marks the plan dirty): seg[t * MMOE_SEG + j] = {src lo, src hi, smem byte offset, prefix
+  // of 16-byte (t = 0, weights) or 4-byte (t = 1, vectors) units}, entry nseg[t] holds the total
+  const uint4* seg;
+  int32_t nseg[2];
 };
 
 }  // namespace souffle
