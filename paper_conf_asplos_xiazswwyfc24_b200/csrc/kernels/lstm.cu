@@ -75,8 +75,11 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
       const int col = v * 16 / ES;   // first element of this vector
       const char* src = col < I ? (const char*)Ly.W + ((int64_t)grow * I + col) * ES
                                 : (const char*)Ly.U + ((int64_t)grow * H + (col - I)) * ES;
-      *reinterpret_cast<uint4*>(w + ((int64_t)r * Kst + col) * ES) = __ldg(reinterpret_cast<const uint4*>(src));
+      // asynchronous copies: every chunk of the tile in flight at once (a load -> store loop waited for
+      // each round trip in turn: ~10 us before the first step)
+      ptx::cp_async16(w + ((int64_t)r * Kst + col) * ES, src);
     }
+    ptx::cp_async_wait_all();
     for (int r = tid; r < R; r += LSTM_THREADS) {
       const int grow = (r / nu) * H + u0 + (r % nu);
       bias[r] = __ldg(Ly.b_ih + grow) + __ldg(Ly.b_hh + grow);
