@@ -99,6 +99,7 @@ __device__ __forceinline__ void bias_chunk(const SwGemm& g, int n, float4* b) {
   for (int c = 0; c < 8; ++c) b[c] = g.bias ? __ldg(reinterpret_cast<const float4*>(g.bias + n) + c) : make_float4(0.f, 0.f, 0.f, 0.f);
 }
 
+template <int EPI>
 __device__ __forceinline__ void epi_chunk(const SwGemm& g, int r, int n, float* v, const float4* bq = nullptr) {
   if (bq) {
 #pragma unroll
@@ -114,17 +115,17 @@ __device__ __forceinline__ void epi_chunk(const SwGemm& g, int r, int n, float* 
       v[c] += b.x; v[c + 1] += b.y; v[c + 2] += b.z; v[c + 3] += b.w;
     }
   }
-  if (g.epi == SWE_F32) {
+  if constexpr (EPI == SWE_F32) {
     float4* dst = reinterpret_cast<float4*>(g.out_f + (int64_t)r * g.N + n);
 #pragma unroll
     for (int c = 0; c < 32; c += 4) dst[c / 4] = make_float4(v[c], v[c + 1], v[c + 2], v[c + 3]);
-  } else if (g.epi == SWE_GELU) {
+  } else if constexpr (EPI == SWE_GELU) {
     uint4* dst = reinterpret_cast<uint4*>(g.out_b + (int64_t)r * g.N + n);
 #pragma unroll
     for (int c = 0; c < 32; c += 8)
       dst[c / 8] = make_uint4(pack_bf16(gelu_erf(v[c]), gelu_erf(v[c + 1])), pack_bf16(gelu_erf(v[c + 2]), gelu_erf(v[c + 3])),
                               pack_bf16(gelu_erf(v[c + 4]), gelu_erf(v[c + 5])), pack_bf16(gelu_erf(v[c + 6]), gelu_erf(v[c + 7])));
-  } else if (g.epi == SWE_RESID) {
+  } else if constexpr (EPI == SWE_RESID) {
     const int tok = g.rowmap ? __ldg(g.rowmap + r) : r;
     float4* xp = reinterpret_cast<float4*>(g.out_f + (int64_t)tok * g.N + n);
     float4 x[8];
@@ -152,11 +153,22 @@ __device__ __forceinline__ void epi_chunk(const SwGemm& g, int r, int n, float* 
   }
 }
 
+// runtime dispatch (the 2-SM kernel serves every epilogue kind)
+__device__ __forceinline__ void epi_chunk_rt(const SwGemm& g, int r, int n, float* v, const float4* bq = nullptr) {
+  switch (g.epi) {
+    case SWE_F32: epi_chunk<SWE_F32>(g, r, n, v, bq); break;
+    case SWE_GELU: epi_chunk<SWE_GELU>(g, r, n, v, bq); break;
+    case SWE_RESID: epi_chunk<SWE_RESID>(g, r, n, v, bq); break;
+    default: epi_chunk<SWE_QKV>(g, r, n, v, bq); break;
+  }
+}
+
 struct GemmCtrl {
   uint64_t full[8], empty[8], tfull[2], tempty[2];
   uint32_t tmem;
 };
 
+template <int EPI>   // the epilogue kind (g.epi): one specialised kernel per fused epilogue
 __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __grid_constant__ GemmArgs A) {
   extern __shared__ __align__(1024) char smem_raw[];
   char* smem = (char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -246,14 +258,37 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       ptx::mbar_wait(&C->tfull[buf], use & 1);
       ptx::tc_fence_after();
       const int rt = q * 32 + lane, r = m0 + rt;
+      if (SP == 1 && EPI == SWE_RESID) {
+        // residual epilogue: the row's destination token (window reverse + roll) once per tile, and
+        // each residual chunk loaded before its accumulator columns are read from TMEM, so the round
+        // trip overlaps the tcgen05.ld (issued after it, it stalled every chunk)
+        const int tok = r < g.M ? (g.rowmap ? __ldg(g.rowmap + r) : r) : 0;
+        for (int c0 = 32 * eh; c0 < BN; c0 += 32 * kEpiGroups) {
+          float v[32];
+          float4 bq[8], x[8];
+          bias_chunk(g, n0 + c0, bq);
+          float4* xp = reinterpret_cast<float4*>(g.out_f + (int64_t)tok * g.N + n0 + c0);
+          if (r < g.M) {
+#pragma unroll
+            for (int c = 0; c < 8; ++c) x[c] = xp[c];
+          }
+          ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
+          if (r < g.M) {
+#pragma unroll
+            for (int c = 0; c < 8; ++c)
+              xp[c] = make_float4(x[c].x + (v[4 * c] + bq[c].x), x[c].y + (v[4 * c + 1] + bq[c].y),
+                                  x[c].z + (v[4 * c + 2] + bq[c].z), x[c].w + (v[4 * c + 3] + bq[c].w));
+          }
+        }
+      } else
       for (int c0 = 32 * eh; c0 < BN; c0 += 32 * kEpiGroups) {
         float v[32];
         float4 bq[8];
         if (SP == 1) bias_chunk(g, n0 + c0, bq);
         ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
         if (SP == 1) {
-          if (r < g.M) epi_chunk(g, r, n0 + c0, v, bq);
-        } else if (g.epi == SWE_RESID) {
+          if (r < g.M) epi_chunk<EPI>(g, r, n0 + c0, v, bq);
+        } else if (EPI == SWE_RESID) {
           // residual epilogue is linear: every split adds its partial (split 0 also the bias)
           // straight into the fp32 residual stream with vector atomics -- no partial round trip
           // (the order of the fp32 adds varies from run to run: ulp-level nondeterminism)
@@ -282,7 +317,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       }
       ptx::tc_fence_before();
       ptx::mbar_arrive(&C->tempty[buf]);
-      if (SP > 1 && g.epi != SWE_RESID) {
+      if (SP > 1 && EPI != SWE_RESID) {
         // meet the other splits of this tile (all units are co-resident: grid == units <= #SMs);
         // the barrier orders every epilogue thread's partial stores before thread et == 0's release
         epi_sync();
@@ -307,7 +342,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
               v[c] += x.x; v[c + 1] += x.y; v[c + 2] += x.z; v[c + 3] += x.w;
             }
           }
-          if (m0 + rr < g.M) epi_chunk(g, m0 + rr, n0 + c0, v);
+          if (m0 + rr < g.M) epi_chunk<EPI>(g, m0 + rr, n0 + c0, v);
         }
         epi_sync();
         if (et == 0) {   // the last split to finish resets the tile's counters for the next run
@@ -477,7 +512,7 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm2_kernel(const __gr
         float4 bq[8];
         bias_chunk(g, n0 + c0, bq);
         ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
-        if (r < g.M) epi_chunk(g, r, n0 + c0, v, bq);
+        if (r < g.M) epi_chunk_rt(g, r, n0 + c0, v, bq);
       }
       ptx::tc_fence_before();
       ptx::mbar_arrive_remote(leader_tempty[buf]);   // the leader's MMA reuses this buffer
@@ -887,9 +922,13 @@ cudaError_t sw_launch_gemm(const void* ta, const void* tb, const SwGemm& g, int 
   memcpy(&a.ta, ta, sizeof(CUtensorMap));
   memcpy(&a.tb, tb, sizeof(CUtensorMap));
   a.g = g;
-  cudaError_t e = set_smem((const void*)swin::sw_gemm_kernel, 227 * 1024);
+  void (*fn)(swin::GemmArgs) = g.epi == SWE_F32    ? swin::sw_gemm_kernel<SWE_F32>
+                               : g.epi == SWE_GELU ? swin::sw_gemm_kernel<SWE_GELU>
+                               : g.epi == SWE_RESID ? swin::sw_gemm_kernel<SWE_RESID>
+                                                    : swin::sw_gemm_kernel<SWE_QKV>;
+  cudaError_t e = set_smem((const void*)fn, 227 * 1024);
   if (e != cudaSuccess) return e;
-  return launch_pdl(swin::sw_gemm_kernel, dim3(grid), dim3(SW_GEMM_THREADS), (size_t)sw_gemm_smem(g.BN, g.stages), s, a);
+  return launch_pdl(fn, dim3(grid), dim3(SW_GEMM_THREADS), (size_t)sw_gemm_smem(g.BN, g.stages), s, a);
 }
 
 cudaError_t sw_launch_gemm2(const void* ta, const void* tb, const SwGemm& g, int grid, cudaStream_t s) {

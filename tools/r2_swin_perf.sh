@@ -1,8 +1,7 @@
 #!/bin/bash
+# Swin pattern: parity + in-graph launch traces at batch 1 / 8 / 64
 mkdir -p gpurun_out
-python -c "from paper_conf_asplos_xiazswwyfc24_b200.build import build; build()" > gpurun_out/build.log 2>&1
-timeout 600 python bench.py --swin-child 0 > gpurun_out/swin_child.json 2> gpurun_out/swin_child.err
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/swin_launches_b64.csv python tools/run_swin_once.py 64 2 > gpurun_out/ncu_swin_l.log 2>&1
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/swin_launches_b1.csv python tools/run_swin_once.py 1 2 > gpurun_out/ncu_swin_l1.log 2>&1
-timeout 900 python -m pytest tests/test_gpu_bert_stages.py -q -m gpu -k ffn1 > gpurun_out/pytest_ffn1.txt 2>&1
+timeout 600 python -m pytest tests/test_gpu_swin.py -q -m gpu > gpurun_out/pytest_swin.txt 2>&1
+echo "rc=$?" >> gpurun_out/pytest_swin.txt
+for b in 1 8 64; do timeout 300 python tools/swin_trace.py $b > gpurun_out/swtrace_b$b.txt 2>&1; done
 echo done
