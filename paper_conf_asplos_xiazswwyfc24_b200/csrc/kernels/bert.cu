@@ -387,15 +387,27 @@ __device__ __forceinline__ void pair_tail(const BertParams& P, const BStage& st,
     v[c] += o.x + b.x; v[c + 1] += o.y + b.y; v[c + 2] += o.z + b.z; v[c + 3] += o.w + b.w;
   }
   const int S = P.S, N = st.N;
+  if (tid == 0) submark(P, st, 9);
   if (st.epi == EP_GELU) {
     if (!(P.dbg_skip & (1 << 22)))   // timing study bit 22: no GELU (wrong values)
 #pragma unroll
       for (int c = 0; c < HC; ++c) v[c] = gelu_erf(v[c]);
-    uint4* dst = reinterpret_cast<uint4*>(st.out_b + (int64_t)row * N + c0);
+    if (tid == 0) submark(P, st, 10);
+    if constexpr (HC == 16) {   // the row's 16 outputs = one 32-byte sector: one 256-bit store
+      uint32_t u[8];
 #pragma unroll
-    for (int c = 0; c < HC; c += 8)
-      dst[c / 8] = make_uint4(pack_bf16(v[c], v[c + 1]), pack_bf16(v[c + 2], v[c + 3]), pack_bf16(v[c + 4], v[c + 5]),
-                              pack_bf16(v[c + 6], v[c + 7]));
+      for (int c = 0; c < 8; ++c) u[c] = pack_bf16(v[2 * c], v[2 * c + 1]);
+      asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(st.out_b + (int64_t)row * N + c0),
+                   "r"(u[0]), "r"(u[1]), "r"(u[2]), "r"(u[3]), "r"(u[4]), "r"(u[5]), "r"(u[6]), "r"(u[7])
+                   : "memory");
+    } else {
+      uint4* dst = reinterpret_cast<uint4*>(st.out_b + (int64_t)row * N + c0);
+#pragma unroll
+      for (int c = 0; c < HC; c += 8)
+        dst[c / 8] = make_uint4(pack_bf16(v[c], v[c + 1]), pack_bf16(v[c + 2], v[c + 3]), pack_bf16(v[c + 4], v[c + 5]),
+                                pack_bf16(v[c + 6], v[c + 7]));
+    }
+    if (tid == 0) submark(P, st, 11);
     return;
   }
   const int H = N / 3;   // EP_QKV (HC columns inside one head)
