@@ -121,7 +121,7 @@ __device__ __forceinline__ void grid_arrive(const BertParams& P, int k, bool tma
   // generic-proxy writes of this stage -> TMA reads of later stages (split-K partials are read by
   // plain loads of the LayerNorm rows: no proxy fence for those stages).  The data is global: the
   // proxy fence is restricted to the global state space (timing study bit 1 << 20: full fence)
-  if (tma_consumed) {
+  if (tma_consumed && !(P.dbg_skip & (1 << 24))) {   // timing study bit 24: no producer-side proxy fence
     if (P.dbg_skip & (1 << 20)) ptx::fence_proxy_async();
     else ptx::fence_proxy_async_global();
   }
