@@ -140,7 +140,12 @@ void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   lp.K_max = std::max(lp.I, lp.H) + lp.H;
   if (lp.K_max > 2 * LSTM_THREADS) return no("input + hidden width above 1024");
   if (lp.L * lp.NP > sms) return no("more CTAs than SMs");
-  if (lstm_smem_bytes(lp.K_max, lp.w_f32) > (size_t)LSTM_MAX_SMEM) return no("weights of 32 units do not fit shared memory");
+  // weights in registers when a CTA's tile fits the register layout (K <= 512, <= 20 units);
+  // SOUFFLE_LSTM_SMEM=1 forces the shared-memory kernel (A/B studies)
+  const int nu_max = (lp.H + lp.NP - 1) / lp.NP;
+  const char* force_smem = std::getenv("SOUFFLE_LSTM_SMEM");
+  lp.reg = (lp.K_max <= LSTM_REG_K && nu_max <= LSTM_REG_UNITS && !(force_smem && std::atoi(force_smem))) ? 1 : 0;
+  if (!lp.reg && lstm_smem_bytes(lp.K_max, lp.w_f32) > (size_t)LSTM_MAX_SMEM) return no("weights of 32 units do not fit shared memory");
   int64_t o = 0;
   lp.o_gen = o; o = al(o + 8, 256);
   lp.o_layers = o; o = al(o + (int64_t)sizeof(LstmLayer) * lp.L, 256);
@@ -159,7 +164,8 @@ std::string lstm_describe(const LstmPlan& lp) {
   }
   os << "pattern lstm: " << lp.L << " layers x " << lp.T << " steps, H=" << lp.H << " I=" << lp.I << " ("
      << (lp.w_f32 ? "fp32" : "bf16") << " weights) -> 1 persistent launch (kernels/lstm.cu), " << lp.L * lp.NP
-     << " CTAs = " << lp.NP << " per layer x <= 32 units, weights resident in shared memory, wavefront of "
+     << " CTAs = " << lp.NP << " per layer x <= " << (lp.H + lp.NP - 1) / lp.NP << " units, weights resident in "
+     << (lp.reg ? "registers (fp32, packed FFMA2 GEMV)" : "shared memory") << ", wavefront of "
      << lp.L + lp.T - 1 << " dependent steps synchronised through tagged (value, step) words\n";
   return os.str();
 }
@@ -214,6 +220,7 @@ souffle_status lstm_run(Plan& p, void* ws, void* stream) {
   prm.NP = lp.NP;
   prm.w_f32 = lp.w_f32;
   prm.K_max = lp.K_max;
+  prm.reg = lp.reg;
   if (p.profiling) {   // debug timeline of one CTA (SOUFFLE_LSTM_PROF_CTA, default the middle layer)
     prm.prof = (unsigned long long*)(base + lp.o_prof);
     const char* e = std::getenv("SOUFFLE_LSTM_PROF_CTA");

@@ -16,6 +16,7 @@ struct LstmPlan {
   bool on = false;
   std::string why_not;
   int T = 0, L = 0, H = 0, I = 0, NP = 0, K_max = 0, w_f32 = 0;
+  int reg = 0;   // 1: register-resident GEMV (lstm_reg_kernel), 0: weights in shared memory
   int X = -1;
   std::vector<int> W, U, bi, bh, h0, c0;   // per layer
   std::vector<int> top;                    // [T] output nodes (last layer h at t)

@@ -214,6 +214,167 @@ __global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_kernel(const __grid_cons
   }
 }
 
+// ---------------------------------------------------------------------------------------------
+// Register-resident variant (K = I + H <= 512 and <= 20 units per CTA, e.g. the 10 x 256 x 100
+// configuration at 14 CTAs per layer): the CTA's 4 nu gate rows are held in fp32 REGISTERS for all
+// T steps (80 weights per thread: 4 nu x 512 x 4 B = 152 KB of the 256 KB register file), so a
+// step's GEMV reads only the 2 KB operand vector from shared memory and issues packed FFMA2s.
+// Warp w owns rows j = 5 (w % 4) + i (i < 5) of gate w / 4; lane q owns columns
+// k = 4 (q + 32 c) + e (c < 4, e < 4: consecutive lanes read consecutive float4s of [x; h], no bank
+// conflicts); the warp's 32 partial sums of each row are combined by a 5-level transpose reduction
+// (8 shuffles), so no cross-warp reduction is needed.  Same dependency protocol and cell as above.
+template <bool F32>
+__global__ void __launch_bounds__(LSTM_THREADS, 1) lstm_reg_kernel(const __grid_constant__ LstmParams P) {
+  __shared__ __align__(16) float xh[LSTM_REG_K];   // [x_t ; h_{t-1}], zero beyond K
+  __shared__ float gates[LSTM_ROWS];
+  __shared__ float bias[LSTM_ROWS];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int l = blockIdx.x / P.NP, p = blockIdx.x % P.NP;
+  const int H = P.H, T = P.T, NP = P.NP;
+  const int u0 = (p * H) / NP, nu = ((p + 1) * H) / NP - u0;   // nu <= 20
+  const LstmLayer& Ly = P.layers[l];
+  const int I = Ly.in_dim, K = I + H;
+  const int gate = warp >> 2, j0 = LSTM_REG_RPW * (warp & 3);   // rows j0 .. j0 + 4 of this gate
+  const bool has_rows = j0 < nu;
+
+  // ---- this thread's 80 weights -> fp32 registers (once for all T steps); zero outside the tile.
+  // I % 8 == 0, so a 4-column group never straddles W_ih | W_hh and its loads are 8 / 16-byte aligned
+  float2 w[LSTM_REG_RPW][4][2];
+#pragma unroll
+  for (int i = 0; i < LSTM_REG_RPW; ++i) {
+    const int j = j0 + i;
+    const int64_t grow = (int64_t)gate * H + u0 + j;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      const int k = 4 * (lane + 32 * c);
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (j < nu && k < K) {
+        const int64_t off = k < I ? grow * I + k : grow * H + (k - I);
+        const void* base = k < I ? Ly.W : Ly.U;
+        if constexpr (F32) {
+          v = __ldg(reinterpret_cast<const float4*>(base) + off / 4);
+        } else {
+          const uint2 u = __ldg(reinterpret_cast<const uint2*>(base) + off / 4);
+          v = make_float4(__uint_as_float(u.x << 16), __uint_as_float(u.x & 0xFFFF0000u), __uint_as_float(u.y << 16),
+                          __uint_as_float(u.y & 0xFFFF0000u));
+        }
+      }
+      w[i][c][0] = make_float2(v.x, v.y);
+      w[i][c][1] = make_float2(v.z, v.w);
+    }
+  }
+  for (int r = tid; r < 4 * nu; r += LSTM_THREADS) {
+    const int grow = (r / nu) * H + u0 + (r % nu);
+    bias[r] = __ldg(Ly.b_ih + grow) + __ldg(Ly.b_hh + grow);
+  }
+  for (int k = tid; k < LSTM_REG_K; k += LSTM_THREADS) xh[k] = 0.f;
+  const int unit = u0 + lane;
+  const bool own = lane < nu;
+  float c = (warp == 0 && own) ? __ldg(Ly.c0 + unit) : 0.f;
+  float h = 0.f;
+  __syncthreads();
+
+  auto stamp = [&](int t, int k) {
+    if (P.prof && blockIdx.x == P.prof_cta && tid == 0) P.prof[4 * t + k] = (unsigned long long)clock64();
+  };
+  const unsigned gen = *(volatile unsigned*)P.gen;
+  const unsigned tag0 = gen * (unsigned)(T + 1) + 1u;
+  for (int t = 0; t < T; ++t) {
+    stamp(t, 0);
+    // ---- [x_t ; h_{t-1}] -> shared memory (thread k fetches element k; K <= 512 threads)
+    if (tid < K) {
+      const int k = tid;
+      if (k < I && l == 0) {
+        xh[k] = __ldg(P.X + (int64_t)t * I + k);
+      } else if (k >= I && t == 0) {
+        xh[k] = __ldg(Ly.h0 + (k - I));
+      } else {
+        const uint2* src = (k < I) ? P.hbuf + ((int64_t)(l - 1) * T + t) * H + k : P.hbuf + ((int64_t)l * T + t - 1) * H + (k - I);
+        const unsigned want = tag0 + (unsigned)(k < I ? t : t - 1);
+        unsigned long long w64;
+        asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w64) : "l"(src) : "memory");
+        while ((unsigned)(w64 >> 32) != want)
+          asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(w64) : "l"(src) : "memory");
+        xh[k] = __uint_as_float((unsigned)w64);
+      }
+    }
+    __syncthreads();
+    stamp(t, 1);
+    // ---- gates: 40 FFMA2 per thread, then the warp's transpose reduction of its 5 row sums
+    if (has_rows) {
+      const float4* x4 = reinterpret_cast<const float4*>(xh);
+      float4 xv[4];
+#pragma unroll
+      for (int cc = 0; cc < 4; ++cc) xv[cc] = x4[lane + 32 * cc];
+      float2 a[LSTM_REG_RPW];
+#pragma unroll
+      for (int i = 0; i < LSTM_REG_RPW; ++i) a[i] = make_float2(0.f, 0.f);
+#pragma unroll
+      for (int cc = 0; cc < 4; ++cc) {
+        const float2 xa = make_float2(xv[cc].x, xv[cc].y), xb = make_float2(xv[cc].z, xv[cc].w);
+#pragma unroll
+        for (int i = 0; i < LSTM_REG_RPW; ++i) {
+          a[i] = __ffma2_rn(w[i][cc][0], xa, a[i]);
+          a[i] = __ffma2_rn(w[i][cc][1], xb, a[i]);
+        }
+      }
+      float v[LSTM_REG_RPW];
+#pragma unroll
+      for (int i = 0; i < LSTM_REG_RPW; ++i) v[i] = a[i].x + a[i].y;
+      // level 1 (xor 16): rows (0, 1, 2) | (3, 4, -); level 2 (xor 8): (u0, u1) | (u2, -);
+      // level 3 (xor 4): one row; levels 4-5 (xor 2, 1): full sums.  Row = 3 b16 + 2 b8 + b4.
+      const bool b16 = lane & 16, b8 = lane & 8, b4 = lane & 4;
+      float u[3];
+#pragma unroll
+      for (int m = 0; m < 3; ++m) {
+        const float lo = v[m], hi = m + 3 < LSTM_REG_RPW ? v[m + 3] : 0.f;
+        u[m] = (b16 ? hi : lo) + __shfl_xor_sync(0xffffffffu, b16 ? lo : hi, 16);
+      }
+      float y[2];
+#pragma unroll
+      for (int m = 0; m < 2; ++m) {
+        const float lo = u[m], hi = m == 0 ? u[2] : 0.f;
+        y[m] = (b8 ? hi : lo) + __shfl_xor_sync(0xffffffffu, b8 ? lo : hi, 8);
+      }
+      float z = (b4 ? y[1] : y[0]) + __shfl_xor_sync(0xffffffffu, b4 ? y[0] : y[1], 4);
+      z += __shfl_xor_sync(0xffffffffu, z, 2);
+      z += __shfl_xor_sync(0xffffffffu, z, 1);
+      const int loc = 2 * (int)b8 + (int)b4, row = 3 * (int)b16 + loc;
+      if ((lane & 3) == 0 && loc < 3 && row < LSTM_REG_RPW && j0 + row < nu) gates[gate * nu + j0 + row] = z;
+    }
+    __syncthreads();
+    stamp(t, 2);
+    // ---- cell update (warp 0, one unit per lane) and publication of h(l, t)
+    if (warp == 0 && own) {
+      const float gi = gates[lane] + bias[lane];
+      const float gf = gates[nu + lane] + bias[nu + lane];
+      const float gg = gates[2 * nu + lane] + bias[2 * nu + lane];
+      const float go = gates[3 * nu + lane] + bias[3 * nu + lane];
+      c = sigm(gf) * c + sigm(gi) * tanh_f(gg);
+      h = sigm(go) * tanh_f(c);
+      if (l == P.L - 1) P.top[t][unit] = h;
+      const unsigned long long w64 = ((unsigned long long)(tag0 + (unsigned)t) << 32) | __float_as_uint(h);
+      uint2* dst = P.hbuf + ((int64_t)l * T + t) * H + unit;
+      asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(dst), "l"(w64) : "memory");
+    }
+    stamp(t, 3);
+  }
+  if (warp == 0 && own) {
+    Ly.h_n[unit] = h;
+    Ly.c_n[unit] = c;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();
+    const unsigned old = atomicAdd(P.gen + 1, 1u);
+    if (old == gridDim.x - 1) {
+      P.gen[1] = 0u;
+      P.gen[0] = gen + 1u;
+      __threadfence();
+    }
+  }
+}
+
 }  // namespace lstm
 
 size_t lstm_smem_bytes(int K_max, int w_f32) {
@@ -221,8 +382,9 @@ size_t lstm_smem_bytes(int K_max, int w_f32) {
 }
 
 cudaError_t lstm_launch(const LstmParams& prm, int grid, cudaStream_t s) {
-  const size_t smem = lstm_smem_bytes(prm.K_max, prm.w_f32);
-  void (*fn)(LstmParams) = prm.w_f32 ? lstm::lstm_kernel<true> : lstm::lstm_kernel<false>;
+  const size_t smem = prm.reg ? 0 : lstm_smem_bytes(prm.K_max, prm.w_f32);
+  void (*fn)(LstmParams) = prm.reg ? (prm.w_f32 ? lstm::lstm_reg_kernel<true> : lstm::lstm_reg_kernel<false>)
+                                   : (prm.w_f32 ? lstm::lstm_kernel<true> : lstm::lstm_kernel<false>);
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg{};

@@ -16,6 +16,9 @@
 namespace souffle {
 
 enum { LSTM_THREADS = 512, LSTM_UNITS = 32, LSTM_ROWS = 4 * LSTM_UNITS, LSTM_MAX_SMEM = 200 * 1024 };
+// register-resident GEMV variant (lstm_reg_kernel): warp w owns rows 5 (w % 4) .. + 4 of gate w / 4 over
+// all K <= 512 columns (16 per lane), so a CTA holds <= 20 units and its weights in fp32 registers
+enum { LSTM_REG_K = 512, LSTM_REG_RPW = 5, LSTM_REG_UNITS = 4 * LSTM_REG_RPW };
 
 struct LstmLayer {
   const void* W;        // W_ih [4H][I_l] (bf16 or fp32, row-major)
@@ -39,7 +42,8 @@ struct LstmParams {
   int32_t w_f32;         // 1: fp32 weights in smem, 0: bf16
   int32_t K_max;         // max_l (I_l + H): row length of the smem weight tile
   unsigned long long* prof;   // debug: per-step timestamps of CTA prof_cta ([T][4]), null if off
-  int32_t prof_cta, pad;
+  int32_t prof_cta;
+  int32_t reg;           // 1: weights resident in registers (lstm_reg_kernel), 0: in shared memory
 };
 
 }  // namespace souffle
