@@ -84,6 +84,28 @@ __device__ __forceinline__ float gelu_erf(float x) {
   const float e = copysignf(1.f - y, u);
   return 0.5f * x * (1.f + e);
 }
+// the same GELU on two values with packed fp32 arithmetic (FFMA2 / FMUL2 / FADD2: every lane's result
+// is the IEEE-rounded scalar result, so the output is bit-identical to gelu_erf; half the issue slots)
+__device__ __forceinline__ float2 gelu_erf2(float2 x) {
+  const float2 u = __fmul2_rn(x, make_float2(0.70710678118654752f, 0.70710678118654752f));
+  const float2 t = make_float2(fminf(fabsf(u.x), 3.92f), fminf(fabsf(u.y), 3.92f));
+  auto cc = [](float c) { return make_float2(c, c); };
+  float2 p = cc(-4.4602740672416985e-05f);
+  p = __ffma2_rn(p, t, cc(4.394397255964577e-04f));
+  p = __ffma2_rn(p, t, cc(-1.4703732449561357e-03f));
+  p = __ffma2_rn(p, t, cc(-8.046277216635644e-04f));
+  p = __ffma2_rn(p, t, cc(2.8278736397624016e-02f));
+  p = __ffma2_rn(p, t, cc(-0.14849244058132172f));
+  p = __ffma2_rn(p, t, cc(-0.9184142351150513f));
+  p = __ffma2_rn(p, t, cc(-1.627908706665039f));
+  const float2 tp = __fmul2_rn(t, p);
+  float2 y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y.x) : "f"(tp.x));
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y.y) : "f"(tp.y));
+  const float2 e = make_float2(copysignf(1.f - y.x, u.x), copysignf(1.f - y.y, u.y));
+  const float2 hx = __fmul2_rn(x, cc(0.5f));
+  return __fmul2_rn(hx, __fadd2_rn(cc(1.f), e));   // (0.5 x)(1 + e), rounded as in gelu_erf
+}
 template <class T>
 __device__ __forceinline__ const void* ldgp(T* const* p) {
   return (const void*)__ldg(reinterpret_cast<const unsigned long long*>(p));
@@ -149,22 +171,26 @@ __device__ __forceinline__ void grid_wait(const BertParams& P, int k, int target
 
 // point-to-point dependency: the producer CTA publishes its epilogue stores (generic proxy -> the
 // consumer's TMA reads) and bumps one flag; the consumer polls only the flag of the data it reads
-__device__ __forceinline__ void flag_signal(const BStage& st, int n0) {
-  ptx::fence_proxy_async();
+__device__ __forceinline__ void flag_signal(const BertParams& P, const BStage& st, int n0) {
+  if (P.dbg_skip & (1 << 25)) ptx::fence_proxy_async();   // timing study bit 25: round-2 fences
+  else ptx::fence_proxy_async_global();                    // the consumer's TMA reads global data
   csync();
   if (threadIdx.x == 0) {
-    __threadfence();
+    // the release below is cumulative over the CTA's writes ordered before it by bar.sync: no
+    // separate gpu-scope fence
+    if (P.dbg_skip & (1 << 25)) __threadfence();
     unsigned* f = st.fout + 32 * ((n0 % st.fmod) / st.fdiv);
     asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(f), "r"(1u) : "memory");
   }
 }
-__device__ __forceinline__ void flag_wait(const BStage& st, int idx) {
+__device__ __forceinline__ void flag_wait(const BertParams& P, const BStage& st, int idx) {
   if (threadIdx.x == 0) {
     const unsigned* f = st.fin + 32 * idx;
     uint32_t n = 0;
     unsigned long long t0 = 0;
     while (ptx::ld_acquire(f) < (unsigned)st.fneed) spin_guard(n, t0);
-    ptx::fence_proxy_async();
+    if (P.dbg_skip & (1 << 25)) ptx::fence_proxy_async();
+    else ptx::fence_proxy_async_global();
   }
   csync();
 }
@@ -389,9 +415,14 @@ __device__ __forceinline__ void pair_tail(const BertParams& P, const BStage& st,
   const int S = P.S, N = st.N;
   if (tid == 0) submark(P, st, 9);
   if (st.epi == EP_GELU) {
-    if (!(P.dbg_skip & (1 << 22)))   // timing study bit 22: no GELU (wrong values)
+    if (!(P.dbg_skip & (1 << 22))) {   // timing study bit 22: no GELU (wrong values)
 #pragma unroll
-      for (int c = 0; c < HC; ++c) v[c] = gelu_erf(v[c]);
+      for (int c = 0; c < HC; c += 2) {
+        const float2 gg = gelu_erf2(make_float2(v[c], v[c + 1]));
+        v[c] = gg.x;
+        v[c + 1] = gg.y;
+      }
+    }
     if (tid == 0) submark(P, st, 10);
     if constexpr (HC == 16) {   // the row's 16 outputs = one 32-byte sector: one 256-bit store
       uint32_t u[8];
@@ -506,7 +537,7 @@ __device__ void run_gemm(const BertParams& P, const BStage& st, Ctrl* C, char* w
     default: gemm_tail<64>(P, st, C, ms, n0, split, areg); break;
   }
   if (tid == 0) submark(P, st, 4);
-  if (st.fout) flag_signal(st, n0);
+  if (st.fout) flag_signal(P, st, n0);
 }
 
 // ------------------------------------------------------------------ attention stage
@@ -819,7 +850,7 @@ __global__ void __launch_bounds__(BERT_THREADS, 1) bert_kernel(const __grid_cons
     const BStage& st = sbuf[s & 1];
     const bool work = has_work(P, st);
     if (work && s > P.s_begin) {
-      if (st.fwait) flag_wait(st, st.kind == BS_ATTN ? (int)blockIdx.x % st.heads : (int)blockIdx.x % st.nsplit);
+      if (st.fwait) flag_wait(P, st, st.kind == BS_ATTN ? (int)blockIdx.x % st.heads : (int)blockIdx.x % st.nsplit);
       else grid_wait(P, s - 1, prev_workers, st.kind != BS_ROW);
     }
     prev_workers = st.workers;
