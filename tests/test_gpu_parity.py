@@ -212,6 +212,30 @@ def test_lstm_ragged_fp32():
     assert rel_err(gs, ws) <= 1e-4
 
 
+@pytest.mark.parametrize("cfg_kw,force_smem", [
+    (dict(steps=6, layers=3, hidden=64, input=64, w_dtype="f32"), True),     # shared-memory kernel, forced
+    (dict(steps=5, layers=2, hidden=320, input=320, w_dtype="bf16"), False),  # K = 640 > 512: shared memory
+    (dict(steps=5, layers=2, hidden=256, input=256, w_dtype="bf16"), True),   # full-width rows, forced
+])
+def test_lstm_shared_memory_kernel(cfg_kw, force_smem, monkeypatch):
+    """The shared-memory LSTM kernel (rows too wide for the register-resident GEMV, or forced with
+    SOUFFLE_LSTM_SMEM=1) stays parity-green next to the register-resident default."""
+    if force_smem:
+        monkeypatch.setenv("SOUFFLE_LSTM_SMEM", "1")
+    cfg = dict(synth.LSTM_CFG, **cfg_kw)
+    gt, wt, gs, ws, plan = _lstm_case(cfg, reps=2)
+    d = plan.describe()
+    assert "weights resident in shared memory" in d, d
+    assert rel_err(gt, wt) <= 1e-4
+    assert rel_err(gs, ws) <= 1e-4
+
+
+def test_lstm_register_kernel_selected():
+    """The default LSTM configuration runs the register-resident GEMV kernel."""
+    _, _, _, _, plan = _lstm_case(dict(synth.LSTM_CFG, steps=3, layers=2), reps=1)
+    assert "weights resident in registers" in plan.describe()
+
+
 def test_lstm_full_config_bf16_weights():
     """BASELINE.json configs[2]: 10 stacked cells, hidden 256, 100 steps, batch 1 (persistent kernel,
     weights resident on chip).  bf16 weights are exact in the oracle; activations stay fp32."""
