@@ -60,7 +60,7 @@ int64_t al(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
 
 }  // namespace
 
-void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, LstmPlan& lp) {
+void lstm_match(const Graph& g, const Analysis& an, const souffle_device_desc& dev, uint32_t flags, LstmPlan& lp) {
   lp = LstmPlan();
   auto no = [&](const char* why) { lp.on = false; lp.why_not = why; };
   if (flags != 0) return no("ablation flags select the generic executor");
@@ -126,6 +126,15 @@ void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, 
   if (g.outputs != expect) return no("outputs are not [top_t..., (h_n, c_n) per layer]");
   lp.hn = h;
   lp.cn = cc;
+  if (an.num_sp != 1) return no("the partition has more than one subprogram");
+  for (size_t i = 0; i < g.nodes.size(); ++i)
+    if (g.nodes[i].op != SOUFFLE_OP_PLACEHOLDER && an.assign[i] != 0) return no("TE outside subprogram 0");
+  // W_hh feeds the dependent chain h(t-1) -> h(t): temporal reuse; W_ih is spatial on layer 0 (its
+  // inputs x_t are independent) and temporal above; either way the T GEMVs share the on-chip copy
+  if (lp.T > 1)
+    for (int n = 0; n < lp.L; ++n)
+      if (an.reuse_kind[lp.W[n]] < 0 || an.reuse_kind[lp.U[n]] != 1)
+        return no("the analysis found no reuse of a layer's weights across the steps (§5.1)");
   // ---- resources: NP CTAs per layer, each owning <= 32 hidden units (<= 128 gate rows) whose
   // weights stay resident in shared memory.  The per-step GEMV is bound by reading those weights
   // from shared memory, so NP is as large as the SMs allow (all layers' CTAs co-resident).

@@ -25,7 +25,10 @@ struct LstmPlan {
   int64_t o_gen = 0, o_layers = 0, o_top = 0, o_hbuf = 0, o_prof = 0, total = 0;
 };
 
-void lstm_match(const Graph& g, const souffle_device_desc& dev, uint32_t flags, LstmPlan& lp);
+// driven by the partition: the analysis must have put every TE in ONE subprogram (Table 5: LSTM runs as
+// one kernel) and found the reuse of every layer's W_ih / W_hh across the T steps (§5.1; W_hh temporal)
+// that the kernel's on-chip weights implement
+void lstm_match(const Graph& g, const Analysis& an, const souffle_device_desc& dev, uint32_t flags, LstmPlan& lp);
 std::string lstm_describe(const LstmPlan& lp);
 
 }  // namespace souffle

@@ -61,7 +61,7 @@ struct Cur {
 };
 }  // namespace
 
-void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
+void mmoe_match(const Graph& g, const Analysis& an, uint32_t flags, MmoePlan& mp) {
   mp = MmoePlan();
   auto no = [&](const char* why) { mp.on = false; mp.why_not = why; };
   if (flags != 0) return no("ablation flags select the generic executor");
@@ -78,12 +78,13 @@ void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
   const int64_t B = mp.B, D = mp.D, De = mp.De;
   Cur c(g);
   c.i = 1;
-  std::vector<int> ex;
+  std::vector<int> ex, xmm;   // xmm: the expert and gate matmuls (all read x)
   // experts: until the first placeholder whose row count differs from De (the first gate)
   while (c.ok && c.i < N.size() && N[c.i].op == SOUFFLE_OP_PLACEHOLDER && N[c.i].shape.size() == 2 &&
          N[c.i].shape[0] == De && N[c.i].shape[1] == D) {
     mp.We.push_back(c.ph({De, D}, wd));
     int m = c.mm(mp.x, mp.We.back());
+    xmm.push_back(m);
     mp.be.push_back(c.ph({De}, SOUFFLE_F32));
     ex.push_back(c.ew(SOUFFLE_EW_RELU, {c.ew(SOUFFLE_EW_ADD, {m, mp.be.back()})}));
   }
@@ -94,6 +95,7 @@ void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
          N[c.i].shape[0] == E && N[c.i].shape[1] == D) {
     mp.Wg.push_back(c.ph({E, D}, wd));
     int m = c.mm(mp.x, mp.Wg.back());
+    xmm.push_back(m);
     mp.bg.push_back(c.ph({E}, SOUFFLE_F32));
     int a = c.ew(SOUFFLE_EW_ADD, {m, mp.bg.back()});
     int mx = c.red(SOUFFLE_RED_MAX, a);
@@ -124,6 +126,15 @@ void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp) {
   }
   if (!c.ok || c.i != N.size()) return no("not an MMoE program (towers)");
   if (g.outputs != mp.y) return no("outputs are not the task towers");
+  if (an.num_sp != 1) return no("the partition has more than one subprogram");
+  for (size_t i = 0; i < g.nodes.size(); ++i)
+    if (g.nodes[i].op != SOUFFLE_OP_PLACEHOLDER && an.assign[i] != 0) return no("TE outside subprogram 0");
+  {
+    const int gid = xmm.empty() || xmm[0] < 0 ? -1 : an.hgid[xmm[0]];
+    bool one = gid >= 0 && an.hkind[gid] == 0;
+    for (int m : xmm) one = one && m >= 0 && an.hgid[m] == gid;
+    if (!one) return no("the analysis did not group the expert and gate matmuls into one N-concat GEMM (§6.1)");
+  }
   if (mp.E > MMOE_MAX_E || mp.T > MMOE_MAX_T || mp.B > MMOE_MAX_B) return no("too many experts / tasks / rows");
   if (mp.B * mp.T > MMOE_THREADS / 32 || mp.Th > 32) return no("batch x tasks > warps or tower width > 32");
   if (1 + mp.E + 3 * mp.T > 32) return no("more than 32 parameter segments (one warp builds the staging table)");

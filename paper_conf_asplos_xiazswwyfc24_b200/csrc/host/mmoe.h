@@ -19,7 +19,9 @@ struct MmoePlan {
   int nseg[2] = {0, 0};   // staging-table segments (set at workspace initialisation)
 };
 
-void mmoe_match(const Graph& g, uint32_t flags, MmoePlan& mp);
+// driven by the partition: ONE subprogram (Table 5), and the expert and gate matmuls that read x form the
+// analysis' N-concat horizontal group (§6.1) that the kernel's fused expert + gate GEMM implements
+void mmoe_match(const Graph& g, const Analysis& an, uint32_t flags, MmoePlan& mp);
 std::string mmoe_describe(const MmoePlan& mp);
 
 }  // namespace souffle

@@ -307,3 +307,26 @@ def test_lstm_gemv_variant_policy(monkeypatch):
     assert "weights resident in shared memory" in describe(layers=2, hidden=320, input=320)
     monkeypatch.setenv("SOUFFLE_LSTM_SMEM", "1")
     assert "weights resident in shared memory" in describe()
+
+
+def test_lstm_and_mmoe_patterns_follow_the_partition():
+    """The LSTM and MMoE pattern lowerings consume the analysis (verdict r1 #4): each program is ONE
+    subprogram run as one launch (Table 5); MMoE's fused expert + gate GEMM is the analysis' N-concat
+    horizontal group of the matmuls that read x (§6.1).  (Both programs are all memory-intensive TEs,
+    so no capacity splits them; the matchers' refusal on a multi-subprogram partition is the BERT
+    matcher's check, exercised above.)"""
+    cases = ((M.lstm, dict(synth.LSTM_CFG, steps=4, layers=3), "pattern lstm: 3 layers"),
+             (M.mmoe, dict(synth.MMOE_CFG), "pattern mmoe:"))
+    for build, cfg, tag in cases:
+        g = build(cfg)[0]
+        plan = g.partition(L.device_b200())
+        d = plan.describe()
+        assert plan.num_subprograms() == 1 and plan.exec_info()["launches"] == 1
+        assert tag in d and "generic lowering: skipped" in d
+        assert g.partition(L.paper_device(1024)).num_subprograms() == 1
+    g = M.mmoe(dict(synth.MMOE_CFG))[0]
+    plan = g.partition(L.device_b200())
+    mm = [i for i in range(plan.num_nodes()) if g.node(i)[0] == L.OP_MATMUL]
+    E, T = synth.MMOE_CFG["experts"], synth.MMOE_CFG["tasks"]
+    groups = {plan.hgroup(i)[1:] for i in mm[:E + T]}
+    assert len(groups) == 1 and next(iter(groups))[1] == 0
