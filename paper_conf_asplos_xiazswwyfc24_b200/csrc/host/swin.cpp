@@ -448,6 +448,7 @@ static souffle_status build_ops(Plan& p, char* base, std::vector<SwinOp>& ops, s
     SwGemm& g = op.gemm;
     std::memset(&g, 0, sizeof(g));
     g.M = (int)M; g.N = (int)N; g.K = (int)K; g.epi = epi;
+    if (const char* e = std::getenv("SOUFFLE_SWIN_EPI_DIRECT")) g.direct = std::atoi(e) != 0;   // A/B studies
     // tile policy: the widest N tile (smem operand bandwidth per MMA) that still fills the SMs;
     // with too few output tiles (small M, e.g. batch 1) the K loop is split across CTAs
     const int64_t mt = (M + 127) / 128, nk = K / 64;

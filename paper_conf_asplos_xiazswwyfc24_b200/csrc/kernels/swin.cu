@@ -189,6 +189,89 @@ __device__ __forceinline__ void epi_chunk_rt(const SwGemm& g, int r, int n, floa
   }
 }
 
+// ---- coalesced epilogue stores through a per-warp 2 KB staging tile (32 rows x 64 bytes).  A warp's
+// accumulator chunk is one row per lane (32 rows x 32 columns); stored straight from registers every
+// store instruction touches 32 rows (32 partial sectors).  Staged, lane l stores 16 bytes of row
+// 8 j + l / 4 (j < 4): 8 rows x 64 contiguous bytes per instruction.  16-byte chunks are XOR-swizzled
+// by row so both the row-per-lane writes and the row-major reads are bank-conflict free.
+constexpr int kEpiStageBytes = 2048;
+__device__ __forceinline__ void stg_put(char* stg, int lane, uint4 a, uint4 b, uint4 c, uint4 d) {
+  const int sw = (lane >> 1) & 3;
+  char* row = stg + lane * 64;
+  *reinterpret_cast<uint4*>(row + ((0 ^ sw) << 4)) = a;
+  *reinterpret_cast<uint4*>(row + ((1 ^ sw) << 4)) = b;
+  *reinterpret_cast<uint4*>(row + ((2 ^ sw) << 4)) = c;
+  *reinterpret_cast<uint4*>(row + ((3 ^ sw) << 4)) = d;
+}
+__device__ __forceinline__ uint4 stg_get(const char* stg, int row, int c) {
+  return *reinterpret_cast<const uint4*>(stg + row * 64 + ((c ^ ((row >> 1) & 3)) << 4));
+}
+__device__ __forceinline__ uint4 f4u(float a, float b, float c, float d) {
+  return make_uint4(__float_as_uint(a), __float_as_uint(b), __float_as_uint(c), __float_as_uint(d));
+}
+
+// one warp's 32 x 32 chunk (rows rbase + lane, columns [n, n + 32)), bias already added, through the
+// staging tile.  RESID: tk[j] is the token row (window reverse + roll) of staged row 8 j + lane / 4 and
+// x[h][j] its residual float4 at column group 16 h + 4 (lane % 4), loaded by the caller before the
+// accumulator so the round trip overlaps the tcgen05.ld.
+template <int EPI>
+__device__ __forceinline__ void epi_staged(const SwGemm& g, int rbase, int lane, int n, const float* v, char* stg,
+                                           const float4 (*x)[4], const int* tk) {
+  const int cq = lane & 3;
+  if constexpr (EPI == SWE_GELU || EPI == SWE_QKV) {
+    // bf16 row of 32 columns = 64 bytes
+    uint32_t u[16];
+    const int which = EPI == SWE_QKV ? n / g.C : 0;
+    const float sc = (EPI == SWE_QKV && which == 0) ? g.qscale : 1.f;
+#pragma unroll
+    for (int c = 0; c < 16; ++c)
+      u[c] = EPI == SWE_GELU ? pack_gelu2(v[2 * c], v[2 * c + 1]) : pack_bf16(v[2 * c] * sc, v[2 * c + 1] * sc);
+    __syncwarp();
+    stg_put(stg, lane, make_uint4(u[0], u[1], u[2], u[3]), make_uint4(u[4], u[5], u[6], u[7]),
+            make_uint4(u[8], u[9], u[10], u[11]), make_uint4(u[12], u[13], u[14], u[15]));
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int row = 8 * j + (lane >> 2), r = rbase + row;
+      if (r >= g.M) continue;
+      const uint4 val = stg_get(stg, row, cq);
+      if constexpr (EPI == SWE_GELU) {
+        *reinterpret_cast<uint4*>(g.out_b + (int64_t)r * g.N + n + 8 * cq) = val;
+      } else {   // Q / K: head-major (window, head) unit rows of 32 bf16
+        const int head = (n % g.C) >> 5, win = r / g.L2, i = r % g.L2;
+        const int64_t unit = (int64_t)win * g.heads + head;
+        *reinterpret_cast<uint4*>((which == 0 ? g.q : g.k) + (unit * SW_WIN_ROWS + i) * 32 + 8 * cq) = val;
+      }
+    }
+  } else {
+    // fp32 rows: two halves of 16 columns (64 bytes)
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const float* w = v + 16 * h;
+      __syncwarp();
+      stg_put(stg, lane, f4u(w[0], w[1], w[2], w[3]), f4u(w[4], w[5], w[6], w[7]), f4u(w[8], w[9], w[10], w[11]),
+              f4u(w[12], w[13], w[14], w[15]));
+      __syncwarp();
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int row = 8 * j + (lane >> 2), r = rbase + row;
+        const uint4 val = stg_get(stg, row, cq);
+        const float4 a = make_float4(__uint_as_float(val.x), __uint_as_float(val.y), __uint_as_float(val.z),
+                                     __uint_as_float(val.w));
+        if constexpr (EPI == SWE_RESID) {
+          if (r < g.M) {
+            const float4 xx = x[h][j];
+            *reinterpret_cast<float4*>(g.out_f + (int64_t)tk[j] * g.N + n + 16 * h + 4 * cq) =
+                make_float4(xx.x + a.x, xx.y + a.y, xx.z + a.z, xx.w + a.w);
+          }
+        } else {
+          if (r < g.M) *reinterpret_cast<float4*>(g.out_f + (int64_t)r * g.N + n + 16 * h + 4 * cq) = a;
+        }
+      }
+    }
+  }
+}
+
 struct GemmCtrl {
   uint64_t full[8], empty[8], tfull[2], tempty[2];
   uint32_t tmem;
@@ -284,7 +367,44 @@ __global__ void __launch_bounds__(SW_GEMM_THREADS, 1) sw_gemm_kernel(const __gri
       ptx::mbar_wait(&C->tfull[buf], use & 1);
       ptx::tc_fence_after();
       const int rt = q * 32 + lane, r = m0 + rt;
-      if (SP == 1 && EPI == SWE_RESID) {
+      if (SP == 1 && !g.direct && EPI != SWE_QKV) {
+        // staged (coalesced) stores (b64: FC1 -9 %, FC2 -13 %, proj -21 %); the QKV scatter keeps the
+        // per-thread stores (each thread's 64-byte Q / K row segment is already whole sectors, and
+        // staging measured +8 %)
+        char* stg = ring + NS * STAGE + (warp - 2) * kEpiStageBytes;
+        const int rbase = m0 + q * 32;
+        int tk[4] = {0, 0, 0, 0};
+        if (EPI == SWE_RESID)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const int rr = rbase + 8 * j + (lane >> 2);
+            tk[j] = rr < g.M ? (g.rowmap ? __ldg(g.rowmap + rr) : rr) : 0;
+          }
+        for (int c0 = 32 * eh; c0 < BN; c0 += 32 * kEpiGroups) {
+          float v[32];
+          float4 bq[8], x[2][4];
+          bias_chunk(g, n0 + c0, bq);
+          if (EPI == SWE_RESID)
+#pragma unroll
+            for (int h = 0; h < 2; ++h)
+#pragma unroll
+              for (int j = 0; j < 4; ++j)
+                x[h][j] = rbase + 8 * j + (lane >> 2) < g.M
+                              ? *reinterpret_cast<const float4*>(g.out_f + (int64_t)tk[j] * g.N + n0 + c0 + 16 * h + 4 * (lane & 3))
+                              : make_float4(0.f, 0.f, 0.f, 0.f);
+          ptx::tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + buf * BN + c0, v);
+          if (EPI == SWE_QKV && (n0 + c0) / g.C == 2) {
+            // V^T: for each column the warp's 32 rows are 64 contiguous bytes already
+            if (r < g.M) epi_chunk<EPI>(g, r, n0 + c0, v, bq);
+          } else {
+#pragma unroll
+            for (int c = 0; c < 8; ++c) {
+              v[4 * c] += bq[c].x; v[4 * c + 1] += bq[c].y; v[4 * c + 2] += bq[c].z; v[4 * c + 3] += bq[c].w;
+            }
+            epi_staged<EPI>(g, rbase, lane, n0 + c0, v, stg, x, tk);
+          }
+        }
+      } else if (SP == 1 && EPI == SWE_RESID) {
         // residual epilogue: the row's destination token (window reverse + roll) once per tile, and
         // each residual chunk loaded before its accumulator columns are read from TMEM, so the round
         // trip overlaps the tcgen05.ld (issued after it, it stalled every chunk)
@@ -941,6 +1061,7 @@ static cudaError_t set_smem(const void* f, int bytes) {
 }
 
 int sw_gemm_smem(int BN, int stages) { return 2048 + stages * (16384 + BN * 128); }
+int sw_gemm1_smem(int BN, int stages) { return sw_gemm_smem(BN, stages) + swin::kEpiWarps * swin::kEpiStageBytes; }
 int sw_attn_smem() { return 2048 + 32768 + 2 * 3 * swin::kAttnTile + swin::kTabBytes; }
 
 cudaError_t sw_launch_gemm(const void* ta, const void* tb, const SwGemm& g, int grid, cudaStream_t s) {
@@ -954,7 +1075,7 @@ cudaError_t sw_launch_gemm(const void* ta, const void* tb, const SwGemm& g, int 
                                                     : swin::sw_gemm_kernel<SWE_QKV>;
   cudaError_t e = set_smem((const void*)fn, 227 * 1024);
   if (e != cudaSuccess) return e;
-  return launch_pdl(fn, dim3(grid), dim3(SW_GEMM_THREADS), (size_t)sw_gemm_smem(g.BN, g.stages), s, a);
+  return launch_pdl(fn, dim3(grid), dim3(SW_GEMM_THREADS), (size_t)sw_gemm1_smem(g.BN, g.stages), s, a);
 }
 
 cudaError_t sw_launch_gemm2(const void* ta, const void* tb, const SwGemm& g, int grid, cudaStream_t s) {

@@ -55,6 +55,7 @@ struct SwGemm {
   unsigned* cnt;
   unsigned long long* trace;  // debug: %globaltimer at the start of launch `op` (CTA 0), or null
   int32_t op;
+  int32_t direct;             // study: 1 = epilogue stores straight from registers (no staging tile)
 };
 
 // window attention over `units` (window, head) pairs, two per CTA iteration.  The additive score

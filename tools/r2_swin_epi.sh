@@ -1,0 +1,10 @@
+#!/bin/bash
+# Swin GEMM epilogue: staged coalesced stores (default) vs per-thread stores (SOUFFLE_SWIN_EPI_DIRECT=1)
+mkdir -p gpurun_out
+timeout 600 python -m pytest tests/test_gpu_swin.py -q -m gpu -x > gpurun_out/pytest_swin.txt 2>&1
+echo "rc=$?" >> gpurun_out/pytest_swin.txt
+for b in 1 8 64; do
+  timeout 300 python tools/swin_trace.py $b > gpurun_out/swe_b$b.txt 2>&1
+  SOUFFLE_SWIN_EPI_DIRECT=1 timeout 300 python tools/swin_trace.py $b > gpurun_out/swd_b$b.txt 2>&1
+done
+echo done
