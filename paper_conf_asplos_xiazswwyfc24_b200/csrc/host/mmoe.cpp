@@ -18,6 +18,7 @@ namespace souffle {
 souffle_status fail(souffle_status c, const std::string& m);
 cudaError_t mmoe_launch(const MmoeParams& prm, cudaStream_t s);
 size_t mmoe_smem_bytes(int B, int D, int E, int De, int T, int Th);
+bool mmoe_cluster_ok(int B, int D, int E, int De, int T);
 
 namespace {
 struct Cur {
@@ -159,8 +160,12 @@ std::string mmoe_describe(const MmoePlan& mp) {
     return os.str();
   }
   os << "pattern mmoe: " << mp.E << " experts x " << mp.De << ", " << mp.T << " tasks, d_in " << mp.D << ", batch "
-     << mp.B << " -> 1 launch (kernels/mmoe.cu): horizontally fused expert+gate GEMM, softmax gates, mixture and "
-        "towers in one CTA, parameters staged once in shared memory\n";
+     << mp.B << " -> 1 launch (kernels/mmoe.cu): horizontally fused expert+gate GEMM, softmax gates, mixture and towers";
+  if (mmoe_cluster_ok(mp.B, mp.D, mp.E, mp.De, mp.T))
+    os << "; cluster of " << MMOE_CL << " CTAs: the fused GEMM split by rows (weights streamed from global memory, "
+          "results to CTA 0 over DSMEM), the rest in CTA 0\n";
+  else
+    os << " in one CTA, parameters staged once in shared memory\n";
   return os.str();
 }
 

@@ -7,7 +7,8 @@
 
 namespace souffle {
 
-enum { MMOE_SEG = 40, MMOE_THREADS = 1024, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
+// MMOE_CL: CTAs of the cluster variant (mmoe_cluster_kernel)
+enum { MMOE_CL = 8, MMOE_SEG = 40, MMOE_THREADS = 1024, MMOE_MAX_E = 16, MMOE_MAX_T = 8, MMOE_MAX_B = 8, MMOE_MAX_SMEM = 200 * 1024 };
 
 struct MmoeParams {
   const float* x;                  // [B][D]

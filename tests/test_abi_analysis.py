@@ -330,3 +330,16 @@ def test_lstm_and_mmoe_patterns_follow_the_partition():
     E, T = synth.MMOE_CFG["experts"], synth.MMOE_CFG["tasks"]
     groups = {plan.hgroup(i)[1:] for i in mm[:E + T]}
     assert len(groups) == 1 and next(iter(groups))[1] == 0
+
+
+def test_mmoe_kernel_variant_policy(monkeypatch):
+    """Host policy of the MMoE lowering: <= 256 fused-GEMM rows (batch x (experts x De + tasks x
+    experts)) and d_in <= 128 run the 8-CTA cluster kernel (rows split over the cluster, DSMEM to CTA 0);
+    larger programs, or SOUFFLE_MMOE_SINGLE=1, the single-CTA kernel."""
+    def describe(**kw):
+        return M.mmoe(dict(synth.MMOE_CFG, **kw))[0].partition(L.device_b200()).describe()
+    assert "cluster of 8 CTAs" in describe()
+    big = dict(batch=4, experts=5, tasks=3, expert_dim=24, tower_hidden=16, d_in=72, w_dtype="bf16")
+    assert "in one CTA" in describe(**big)
+    monkeypatch.setenv("SOUFFLE_MMOE_SINGLE", "1")
+    assert "in one CTA" in describe()

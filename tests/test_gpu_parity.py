@@ -163,6 +163,26 @@ def test_mmoe(cfg, flags, record_err):
         record_err(rel_err(r, ref[o]), 1e-4)
 
 
+def test_mmoe_single_cta_kernel(monkeypatch, record_err):
+    """The single-CTA MMoE kernel on the default configuration (the cluster kernel's shape), forced with
+    SOUFFLE_MMOE_SINGLE=1; test_mmoe covers the cluster kernel (default) and the single kernel (batch 4)."""
+    monkeypatch.setenv("SOUFFLE_MMOE_SINGLE", "1")
+    cfg = synth.MMOE_CFG
+    p = synth.mmoe_params(cfg)
+    x = synth.mmoe_input(cfg)
+    spec, names, outs = og.mmoe(cfg)
+    feed = {names[k]: v for k, v in p.items()}
+    feed[names["x"]] = x
+    ref = te.evaluate(spec, feed)
+    g, gn, gouts = M.mmoe(cfg)
+    gfeed = {gn[k]: v for k, v in p.items()}
+    gfeed[gn["x"]] = x
+    res, plan = run(g, gfeed, gouts, 0)
+    assert "in one CTA" in plan.describe()
+    for o, r in zip(outs, res):
+        record_err(rel_err(r, ref[o]), 1e-4)
+
+
 def _lstm_case(cfg, flags=0, reps=1):
     x = synth.lstm_input(cfg)
     ps = synth.lstm_params(cfg)
