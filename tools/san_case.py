@@ -1,5 +1,6 @@
 """One small launch of a kernel family, checked against the oracle (for compute-sanitizer runs).
-usage: python tools/san_case.py bert_small | swin_small | generic_tiny | rowwise | swin_generic | mbconv:IDX
+usage: python tools/san_case.py bert_small | swin_small | generic_tiny | rowwise | swin_generic | mbconv:IDX |
+       lstm_small | mmoe
 (rowwise / swin_generic / generic_tiny exercise the generic executor's row-block stages and tensor cache;
 SOUFFLE_CACHE_FLOATS=2048 forces LRU spills)"""
 import os
@@ -39,6 +40,42 @@ elif which.startswith("mbconv:"):
     s.run()
     s.run()
     out = s.result(gy)
+elif which in ("lstm_small", "mmoe"):
+    if which == "lstm_small":   # register-resident GEMV kernel (3 layers x 64 units x 5 steps)
+        cfg = dict(synth.LSTM_CFG, steps=5, layers=3, hidden=64, input=64, w_dtype="f32")
+        x, ps = synth.lstm_input(cfg), synth.lstm_params(cfg)
+        spec, names, top, hs, cs = og.lstm(cfg)
+
+        def feed_for(nm):
+            f = {nm["X"]: x}
+            for n, q in enumerate(ps):
+                f[nm[f"W{n}"]], f[nm[f"U{n}"]] = q["W"], q["U"]
+                f[nm[f"bih{n}"]], f[nm[f"bhh{n}"]] = q["b_ih"], q["b_hh"]
+                f[nm[f"h0_{n}"]] = np.zeros((1, cfg["hidden"]), np.float32)
+                f[nm[f"c0_{n}"]] = np.zeros((1, cfg["hidden"]), np.float32)
+            return f
+        ref = te.evaluate(spec, feed_for(names))[top[-1]]
+        g, gn, gtop, ghs, gcs = M.lstm(cfg)
+        plan = g.partition(L.device_query(0))
+        s = session(g, plan, feed_for(gn), [gtop[-1]])
+        s.run()
+        s.run()
+        out = s.result(gtop[-1])
+    else:                       # 8-CTA cluster kernel
+        cfg = synth.MMOE_CFG
+        p, x = synth.mmoe_params(cfg), synth.mmoe_input(cfg)
+        spec, names, outs = og.mmoe(cfg)
+        feed = {names[k]: v for k, v in p.items()}
+        feed[names["x"]] = x
+        ref = te.evaluate(spec, feed)[outs[0]]
+        g, gn, gouts = M.mmoe(cfg)
+        gfeed = {gn[k]: v for k, v in p.items()}
+        gfeed[gn["x"]] = x
+        plan = g.partition(L.device_query(0))
+        s = session(g, plan, gfeed, gouts)
+        s.run()
+        out = s.result(gouts[0])
+    print(plan.describe().splitlines()[1 if which == "lstm_small" else 2][:160])
 elif which == "rowwise":
     spec = synth.random_rowwise_spec(0)
     ins = synth.spec_inputs(spec, 0)
