@@ -503,3 +503,65 @@ def mbconv(cfg):
 def synth_dims(cfg):
     """exp, squeeze of an MBConv config (torchvision: squeeze = max(1, cin // 4))."""
     return dict(exp=cfg["cin"] * cfg["expand"], squeeze=max(1, cfg["cin"] // 4))
+
+
+def resnext(cfg):
+    """ResNeXt Bottleneck block (Table 2: ResNeXt-101, 64 groups x 4d; torchvision
+    resnext101_64x4d Bottleneck in inference form) as a TE program over NHWC, batch 1:
+      a = ReLU(BN(x W1^T))                                1x1 convolution to the bottleneck width
+      c = sum_t  m_t * roll(a, -o_t)  grouped by G:        the 3x3 grouped convolution, zero padding 1:
+          [HW, G, cg] -> [G, HW, cg] (x) W2_t [G, cg, cg]^T  tap t reads a shifted by its offset o_t (a
+                                                          roll TE, border mask m_t) and every group g
+                                                          multiplies its cg channels by W2_t[g] -- ONE
+                                                          batched matmul TE per tap over the G groups
+      d = ReLU(BN(c[::s, ::s]))
+      y = ReLU(BN(d W3^T) + shortcut),  shortcut = x, or BN(x[::s, ::s] Wd^T) when the shape changes
+    BN is the per-channel affine y = x * s + b.  Returns (spec, names, x id, y id)."""
+    H, s, G = cfg["hw"], cfg["stride"], cfg["groups"]
+    cin, w, cout = cfg["cin"], cfg["width"], cfg["cout"]
+    cg, Ho = w // G, H // s
+    b = SpecBuilder()
+    names = {}
+    x = b.ph((H * H, cin), const=0)
+    names["W1"] = b.ph((w, cin))
+    a = b.mm(x, names["W1"], 1, "f32")
+    names["s1"], names["b1"] = b.ph((w,)), b.ph((w,))
+    a = b.ew("relu", b.ew("add", b.ew("mul", a, names["s1"]), names["b1"]))
+    a3 = b.reshape(a, (H, H, w))
+    acc = None
+    for i in range(3):
+        for j in range(3):
+            t = i * 3 + j
+            if i == 1 and j == 1:
+                term = a3
+            else:
+                r = b._add({"op": "roll", "in": a3, "shifts": [1 - i, 1 - j, 0]})   # r[h, w] = a[h + i - 1, w + j - 1]
+                names[f"m{t}"] = b.ph((H, H, 1))
+                term = b.ew("mul", r, names[f"m{t}"])
+            tg = b.permute(b.reshape(term, (H * H, G, cg)), (1, 0, 2))           # [G, HW, cg]
+            names[f"W2_{t}"] = b.ph((G, cg, cg))
+            pt = b.mm(tg, names[f"W2_{t}"], 1, "f32")                             # [G, HW, cg]
+            acc = pt if acc is None else b.ew("add", acc, pt)
+    c3 = b.reshape(b.permute(acc, (1, 0, 2)), (H, H, w))
+    if s != 1:
+        c3 = b.slice(c3, (0, 0, 0), (H, H, w), (s, s, 1))
+    d = b.reshape(c3, (Ho * Ho, w))
+    names["s2"], names["b2"] = b.ph((w,)), b.ph((w,))
+    d = b.ew("relu", b.ew("add", b.ew("mul", d, names["s2"]), names["b2"]))
+    names["W3"] = b.ph((cout, w))
+    y = b.mm(d, names["W3"], 1, "f32")
+    names["s3"], names["b3"] = b.ph((cout,)), b.ph((cout,))
+    y = b.ew("add", b.ew("mul", y, names["s3"]), names["b3"])
+    if s != 1 or cin != cout:
+        xs = x
+        if s != 1:
+            xs = b.reshape(b.slice(b.reshape(x, (H, H, cin)), (0, 0, 0), (H, H, cin), (s, s, 1)), (Ho * Ho, cin))
+        names["Wd"] = b.ph((cout, cin))
+        sc = b.mm(xs, names["Wd"], 1, "f32")
+        names["sd"], names["bd"] = b.ph((cout,)), b.ph((cout,))
+        sc = b.ew("add", b.ew("mul", sc, names["sd"]), names["bd"])
+    else:
+        sc = x
+    y = b.ew("relu", b.ew("add", y, sc))
+    b.out(y)
+    return b.spec(), names, x, y

@@ -400,3 +400,58 @@ def mbconv(cfg):
         y = g.ew("add", y, x)
     g.mark_output(y)
     return g, names, x, y
+
+
+def resnext(cfg):
+    """ResNeXt Bottleneck block (Table 2: ResNeXt-101, 64 groups x 4d) as a TE program (same
+    node order as oracle.graphs.resnext): 1x1 convolutions as matmuls, the grouped 3x3 convolution as
+    rolled + border-masked taps, each one batched matmul over the groups; BatchNorm as a per-channel
+    affine; x [H*W, Cin] NHWC, batch 1.  Returns (graph, names, x, y)."""
+    H, s, G = cfg["hw"], cfg["stride"], cfg["groups"]
+    cin, w, cout = cfg["cin"], cfg["width"], cfg["cout"]
+    cg, Ho = w // G, H // s
+    g = L.Graph()
+    names = {}
+    x = g.placeholder((H * H, cin), L.F32, const=False)
+    names["W1"] = g.placeholder((w, cin))
+    a = g.matmul(x, names["W1"], True, L.F32)
+    names["s1"], names["b1"] = g.placeholder((w,)), g.placeholder((w,))
+    a = g.ew("relu", g.ew("add", g.ew("mul", a, names["s1"]), names["b1"]))
+    a3 = g.reshape(a, (H, H, w))
+    acc = None
+    for i in range(3):
+        for j in range(3):
+            t = i * 3 + j
+            if i == 1 and j == 1:
+                term = a3
+            else:
+                r = g.roll(a3, (1 - i, 1 - j, 0))
+                names[f"m{t}"] = g.placeholder((H, H, 1))
+                term = g.ew("mul", r, names[f"m{t}"])
+            tg = g.permute(g.reshape(term, (H * H, G, cg)), (1, 0, 2))
+            names[f"W2_{t}"] = g.placeholder((G, cg, cg))
+            pt = g.matmul(tg, names[f"W2_{t}"], True, L.F32)
+            acc = pt if acc is None else g.ew("add", acc, pt)
+    c3 = g.reshape(g.permute(acc, (1, 0, 2)), (H, H, w))
+    if s != 1:
+        c3 = g.slice(c3, (0, 0, 0), (H, H, w), (s, s, 1))
+    d = g.reshape(c3, (Ho * Ho, w))
+    names["s2"], names["b2"] = g.placeholder((w,)), g.placeholder((w,))
+    d = g.ew("relu", g.ew("add", g.ew("mul", d, names["s2"]), names["b2"]))
+    names["W3"] = g.placeholder((cout, w))
+    y = g.matmul(d, names["W3"], True, L.F32)
+    names["s3"], names["b3"] = g.placeholder((cout,)), g.placeholder((cout,))
+    y = g.ew("add", g.ew("mul", y, names["s3"]), names["b3"])
+    if s != 1 or cin != cout:
+        xs = x
+        if s != 1:
+            xs = g.reshape(g.slice(g.reshape(x, (H, H, cin)), (0, 0, 0), (H, H, cin), (s, s, 1)), (Ho * Ho, cin))
+        names["Wd"] = g.placeholder((cout, cin))
+        sc = g.matmul(xs, names["Wd"], True, L.F32)
+        names["sd"], names["bd"] = g.placeholder((cout,)), g.placeholder((cout,))
+        sc = g.ew("add", g.ew("mul", sc, names["sd"]), names["bd"])
+    else:
+        sc = x
+    y = g.ew("relu", g.ew("add", y, sc))
+    g.mark_output(y)
+    return g, names, x, y

@@ -347,3 +347,51 @@ def mbconv_masks(cfg: dict) -> dict:
             mw = ((h + j - pad) >= 0) & ((h + j - pad) < H)
             out[f"m{i * k + j}"] = (mh[:, None] & mw[None, :]).astype(np.float32).reshape(H, H, 1)
     return out
+
+
+# ---------------------------------------------------------------- ResNeXt bottleneck blocks R0-R7
+# PAPER.md Table 2 (L1303): ResNeXt-101 with 64 groups x 4d bottleneck width (torchvision
+# resnext101_64x4d: groups 64, width_per_group 4, layers [3, 4, 23, 3], stride on the grouped 3x3
+# convolution).  Its distinct Bottleneck shapes: the first block of each stage (projection shortcut,
+# stride 2 from stage 2 on) and the repeated identity block, batch 1, NHWC.
+RESNEXT_CONFIGS = [
+    dict(name=f"R{i}", cin=ci, width=w, cout=co, hw=h, stride=s, groups=64)
+    for i, (ci, w, co, h, s) in enumerate([
+        (64, 256, 256, 56, 1), (256, 256, 256, 56, 1), (256, 512, 512, 56, 2), (512, 512, 512, 28, 1),
+        (512, 1024, 1024, 28, 2), (1024, 1024, 1024, 14, 1), (1024, 2048, 2048, 14, 2), (2048, 2048, 2048, 7, 1)])
+]
+
+
+def resnext_projection(cfg: dict) -> bool:
+    """torchvision: a 1x1 (strided) convolution + BN on the shortcut when the shape changes."""
+    return cfg["stride"] != 1 or cfg["cin"] != cfg["cout"]
+
+
+def resnext_input(cfg: dict, seed: int = INPUT_SEED) -> np.ndarray:
+    """x [H*W, Cin] fp32 ~ N(0, 1) (NHWC, batch 1)."""
+    return normal(seed, (cfg["hw"] * cfg["hw"], cfg["cin"]))
+
+
+def resnext_params(cfg: dict) -> dict:
+    """Random-init weights of one Bottleneck (BatchNorm in inference form: y = x * s + b).  1x1
+    convolutions as [out, in] matrices; the grouped 3x3 convolution as one [G, cg_out, cg_in] tensor per
+    tap t = i * 3 + j (group g's [cg_out, cg_in] slice of torch's weight[:, :, i, j]); fp32."""
+    cin, w, cout, G = cfg["cin"], cfg["width"], cfg["cout"], cfg["groups"]
+    cg = w // G
+    base = 5000 + cfg["cin"] + 7 * cfg["hw"]
+    p = dict(W1=normal(base + 1, (w, cin), std=1.0 / np.sqrt(cin)), s1=normal(base + 2, (w,), std=0.1, mean=1.0),
+             b1=normal(base + 3, (w,), std=0.1))
+    for t in range(9):
+        p[f"W2_{t}"] = normal(base + 10 + t, (G, cg, cg), std=1.0 / np.sqrt(9 * cg))
+    p.update(s2=normal(base + 4, (w,), std=0.1, mean=1.0), b2=normal(base + 5, (w,), std=0.1),
+             W3=normal(base + 6, (cout, w), std=1.0 / np.sqrt(w)), s3=normal(base + 7, (cout,), std=0.1, mean=1.0),
+             b3=normal(base + 8, (cout,), std=0.1))
+    if resnext_projection(cfg):
+        p.update(Wd=normal(base + 30, (cout, cin), std=1.0 / np.sqrt(cin)), sd=normal(base + 31, (cout,), std=0.1, mean=1.0),
+                 bd=normal(base + 32, (cout,), std=0.1))
+    return p
+
+
+def resnext_masks(cfg: dict) -> dict:
+    """Zero padding of the 3x3 convolution as data (the border masks of mbconv_masks with k = 3)."""
+    return mbconv_masks(dict(hw=cfg["hw"], k=3))
