@@ -11,8 +11,8 @@ LIB = os.path.join(HERE, "libsouffle.so")
 ROOT = os.path.dirname(HERE)
 
 SOURCES = [
-    "host/analysis.cpp", "host/lower.cpp", "host/api.cpp", "host/runtime.cpp", "host/bert.cpp", "host/lstm.cpp", "host/mmoe.cpp", "host/swin.cpp", "host/se.cpp", "host/mbconv.cpp",
-    "kernels/exec.cu", "kernels/bert.cu", "kernels/lstm.cu", "kernels/mmoe.cu", "kernels/swin.cu", "kernels/se.cu", "kernels/mbconv.cu",
+    "host/analysis.cpp", "host/lower.cpp", "host/api.cpp", "host/runtime.cpp", "host/bert.cpp", "host/lstm.cpp", "host/mmoe.cpp", "host/swin.cpp", "host/se.cpp", "host/mbconv.cpp", "host/resnext.cpp",
+    "kernels/exec.cu", "kernels/bert.cu", "kernels/lstm.cu", "kernels/mmoe.cu", "kernels/swin.cu", "kernels/se.cu", "kernels/mbconv.cu", "kernels/resnext.cu",
 ]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",

@@ -496,6 +496,12 @@ souffle_status souffle_plan_exec_info(souffle_plan p, int32_t* launches, int32_t
       if (barriers) *barriers = 3;
       return;
     }
+    if (P.rx.on) {   // 1x1 (+ projection) | grouped 3x3 | 1x1 + shortcut
+      if (launches) *launches = 1;
+      if (stages) *stages = 3;
+      if (barriers) *barriers = 2;
+      return;
+    }
     if (P.swin.on) {   // one kernel per fused subprogram, replayed as one CUDA graph
       if (launches) *launches = P.swin.launches;
       if (stages) *stages = P.swin.launches;

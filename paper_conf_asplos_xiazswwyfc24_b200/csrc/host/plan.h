@@ -11,6 +11,7 @@
 #include "swin.h"
 #include "se.h"
 #include "mbconv.h"
+#include "resnext.h"
 #include "ir.h"
 
 namespace souffle {
@@ -66,6 +67,7 @@ struct Plan {
   SwinPlan swin;                    // pattern lowering (swin.on: kernels/swin.cu, one CUDA graph)
   SePlan se;                        // pattern lowering (se.on: kernels/se.cu, EfficientNet M0-M9)
   MbPlan mb;                        // pattern lowering (mb.on: kernels/mbconv.cu, MBConv blocks M0-M9)
+  RxPlan rx;                        // pattern lowering (rx.on: kernels/resnext.cu, ResNeXt blocks R0-R7)
   ~Plan();
 };
 

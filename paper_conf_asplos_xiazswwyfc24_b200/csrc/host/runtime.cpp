@@ -31,6 +31,7 @@ souffle_status swin_init(Plan& p, void* ws, void* stream);
 souffle_status swin_run(Plan& p, void* ws, void* stream);
 souffle_status se_run(Plan& p, void* ws, void* stream);
 souffle_status mbconv_run(Plan& p, void* ws, void* stream);
+souffle_status resnext_run(Plan& p, void* ws, void* stream);
 souffle_status mmoe_init(Plan& p, void* ws, void* stream);
 
 size_t workspace_bytes(Plan& p) {
@@ -40,6 +41,7 @@ size_t workspace_bytes(Plan& p) {
   if (p.swin.on) return (size_t)p.swin.total;
   if (p.se.on) return (size_t)p.se.total;
   if (p.mb.on) return (size_t)p.mb.total;
+  if (p.rx.on) return (size_t)p.rx.total;
   WsLayout& w = p.ws;
   w.ctrl_off = 0;
   // barrier words + stage timestamps + 8 sub-stage marks per stage
@@ -113,8 +115,8 @@ souffle_status init_workspace(Plan& p, void* ws, void* stream) {
   if (p.bert.on) return bert_init(p, ws, stream);
   if (p.lstm.on) return lstm_init(p, ws, stream);
   if (p.swin.on) return swin_init(p, ws, stream);
-  if (p.se.on || p.mb.on) {   // barrier counters start at zero (the last CTA of every launch resets them)
-    cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)(p.se.on ? p.se.total : p.mb.total), (cudaStream_t)stream);
+  if (p.se.on || p.mb.on || p.rx.on) {   // barrier counters start at zero (the last CTA of every launch resets them)
+    cudaError_t e = cudaMemsetAsync(ws, 0, (size_t)(p.se.on ? p.se.total : p.mb.on ? p.mb.total : p.rx.total), (cudaStream_t)stream);
     if (e != cudaSuccess) return fail(SOUFFLE_E_CUDA, std::string("se workspace init: ") + cudaGetErrorString(e));
     p.inited_ws = ws;
     p.dirty = false;
@@ -205,6 +207,11 @@ souffle_status run_plan(Plan& p, void* ws, void* stream) {
     std::string why;
     if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
     return mbconv_run(p, ws, stream);
+  }
+  if (p.rx.on) {
+    std::string why;
+    if (!device_ok(why)) return fail(SOUFFLE_E_UNSUPPORTED, why);
+    return resnext_run(p, ws, stream);
   }
   static int max_active = -1;
   if (max_active < 0) {

@@ -1,0 +1,206 @@
+// ResNeXt Bottleneck block (Table 2: ResNeXt-101, 64 groups x 4d) as ONE persistent kernel on
+// sm_100a (the TE program of csrc/resnext_types.h, fp32 like the oracle):
+//
+//   1  a = ReLU(x W1^T * s1 + b1)                 64 x 64 (or 32 x 32) tiles over the grid, and the
+//      projection shortcut y = x[::s, ::s] Wd^T * sd + bd (when the shape changes)        | sync
+//   2  d = ReLU(sum_t m_t[p] sum_i W2_t[g][o][i] a[p + o_t][g cg + i] * s2 + b2) at the strided output
+//      pixels: the grouped 3x3 convolution; the TE's roll is a cyclic shift, so tap t reads a at
+//      ((h + i - 1) mod H, (w + j - 1) mod H) and the border mask (an input) zeroes what wrapped
+//      around; one thread per (pixel, output channel), float4 loads along the group's channels | sync
+//   3  y = ReLU(d W3^T * s3 + b3 + shortcut)       (shortcut: x, or the projection from phase 1)
+//
+// Two grid synchronisations -- the one-relies-on-many dependencies of the block (the 3x3 halo needs
+// neighbouring pixels of a, the second 1x1 convolution every channel of d) -- and no other launch.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../resnext_types.h"
+#include "ptx.cuh"
+
+namespace souffle {
+namespace rx {
+
+__device__ __forceinline__ void grid_sync(const RxParams& P, int k) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    ptx::red_release_add(&P.ctrl[k], 1u);
+    while (ptx::ld_acquire(&P.ctrl[k]) < gridDim.x) {
+    }
+  }
+  __syncthreads();
+}
+__device__ __forceinline__ void stamp(const RxParams& P, int k) {
+  if (P.prof && blockIdx.x == 0 && threadIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    P.prof[k] = t;
+  }
+}
+// L1-cached load of data written earlier in this launch by other CTAs: safe after the grid barrier (its
+// acquire invalidates L1, and the data is not written again); the 3x3 taps re-read a up to 9 times
+__device__ __forceinline__ float4 ld_ca4(const float* p) {
+  float4 v;
+  asm volatile("ld.global.ca.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+  return v;
+}
+
+// C[m0.., n0..] (BM x BN) = sum_k A(arow(m), k) B[n][k]; epi(m, n, v) for the in-range outputs.  256
+// threads, (BM/16) x (BN/16) outputs each; K in slabs of 16 staged k-major in shared memory.
+template <int BM, int BN, class Row, class Epi>
+__device__ __forceinline__ void tile(const float* A, int lda, Row arow, const float* B, int M, int N, int K, int m0,
+                                     int n0, float* sm, Epi epi) {
+  constexpr int RM = BM / 16, RN = BN / 16;
+  float(*As)[BM + 1] = reinterpret_cast<float(*)[BM + 1]>(sm);
+  float(*Bs)[BN + 1] = reinterpret_cast<float(*)[BN + 1]>(sm + 16 * (BM + 1));
+  const int tid = threadIdx.x, ty = tid >> 4, tx = tid & 15;
+  float c[RM][RN];
+#pragma unroll
+  for (int i = 0; i < RM; ++i)
+#pragma unroll
+    for (int j = 0; j < RN; ++j) c[i][j] = 0.f;
+  for (int k0 = 0; k0 < K; k0 += 16) {
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < (BM * 16) / RX_THREADS; ++q) {
+      const int e = tid + q * RX_THREADS, kk = e & 15, r = e >> 4, k = k0 + kk;
+      As[kk][r] = (m0 + r < M && k < K) ? __ldcg(A + (int64_t)arow(m0 + r) * lda + k) : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < (BN * 16) / RX_THREADS; ++q) {
+      const int e = tid + q * RX_THREADS, kk = e & 15, r = e >> 4, k = k0 + kk;
+      Bs[kk][r] = (n0 + r < N && k < K) ? __ldg(B + (int64_t)(n0 + r) * K + k) : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < 16; ++kk) {
+      float av[RM], bv[RN];
+#pragma unroll
+      for (int i = 0; i < RM; ++i) av[i] = As[kk][ty * RM + i];
+#pragma unroll
+      for (int j = 0; j < RN; ++j) bv[j] = Bs[kk][tx * RN + j];
+#pragma unroll
+      for (int i = 0; i < RM; ++i)
+#pragma unroll
+        for (int j = 0; j < RN; ++j) c[i][j] = fmaf(av[i], bv[j], c[i][j]);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < RM; ++i)
+#pragma unroll
+    for (int j = 0; j < RN; ++j) {
+      const int m = m0 + ty * RM + i, n = n0 + tx * RN + j;
+      if (m < M && n < N) epi(m, n, c[i][j]);
+    }
+}
+
+// the tiles of one GEMM, task t0.. of a shared task space: 64 x 64 tiles when they fill half the grid,
+// else 32 x 32.  Returns the number of tasks it has.
+template <class Row, class Epi>
+__device__ __forceinline__ int gemm_tasks(const float* A, int lda, Row arow, const float* B, int M, int N, int K,
+                                          int t0, float* sm, Epi epi) {
+  const int t64 = ((M + 63) / 64) * ((N + 63) / 64);
+  const bool big = 2 * t64 >= (int)gridDim.x;
+  const int bm = big ? 64 : 32, tn = (N + bm - 1) / bm, nt = ((M + bm - 1) / bm) * tn;
+  for (int t = (int)blockIdx.x - t0; t < nt; t += gridDim.x) {
+    if (t < 0) continue;
+    if (big) tile<64, 64>(A, lda, arow, B, M, N, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
+    else tile<32, 32>(A, lda, arow, B, M, N, K, (t / tn) * 32, (t % tn) * 32, sm, epi);
+  }
+  return nt;
+}
+
+template <int CG>   // channels per group (0: any, loops not unrolled)
+__global__ void __launch_bounds__(RX_THREADS, 1) resnext_kernel(const __grid_constant__ RxParams P) {
+  __shared__ float tsm[2 * 16 * 65];   // GEMM operand slabs
+  const int tid = threadIdx.x;
+  const int H = P.H, w = P.w, s = P.stride, cout = P.cout, cin = P.cin;
+  const int HW = H * H, Ho = H / s, HWo = Ho * Ho;
+  const int cg = CG ? CG : w / P.G;
+  auto ident = [](int m) { return m; };
+
+  stamp(P, 0);
+  // ---- 1: 1x1 convolution (+ BN + ReLU), and the projection shortcut into y (its tasks continue the
+  // task numbering so the two GEMMs share the grid)
+  const int n1 = gemm_tasks(P.x, cin, ident, P.W1, HW, w, cin, 0, tsm, [&](int m, int n, float v) {
+    P.a[(int64_t)m * w + n] = fmaxf(v * __ldg(P.s1 + n) + __ldg(P.b1 + n), 0.f);
+  });
+  if (P.Wd) {
+    auto srow = [&](int m) { return (m / Ho) * s * H + (m % Ho) * s; };   // output pixel -> input row
+    gemm_tasks(P.x, cin, srow, P.Wd, HWo, cout, cin, n1 % (int)gridDim.x, tsm, [&](int m, int n, float v) {
+      P.y[(int64_t)m * cout + n] = v * __ldg(P.sd + n) + __ldg(P.bd + n);
+    });
+  }
+  stamp(P, 1);
+  grid_sync(P, 0);
+  // ---- 2: grouped 3x3 convolution (+ BN + ReLU) at the strided output pixels; (pixel, channel) pairs
+  // spread over the grid, consecutive threads = consecutive output channels
+  {
+    const int64_t total = (int64_t)HWo * w;
+    for (int64_t idx = (int64_t)blockIdx.x * RX_THREADS + tid; idx < total; idx += (int64_t)gridDim.x * RX_THREADS) {
+      const int q = (int)(idx / w), o = (int)(idx % w);
+      const int g = o / cg, oo = o % cg;
+      const int hs = (q / Ho) * s, ws = (q % Ho) * s;   // the pixel in the stride-1 grid
+      float acc = 0.f;
+#pragma unroll
+      for (int t = 0; t < RX_TAPS; ++t) {
+        const int i = t / 3, j = t % 3;
+        const int hh = (hs + i - 1 + H) % H, ww = (ws + j - 1 + H) % H;
+        const float* ar = P.a + (int64_t)(hh * H + ww) * w + g * cg;
+        const float* wr = P.W2[t] + ((int64_t)g * cg + oo) * cg;
+        float part = 0.f;
+#pragma unroll 4
+        for (int ii = 0; ii < cg; ii += 4) {
+          const float4 av = ld_ca4(ar + ii);
+          const float4 wv = __ldg(reinterpret_cast<const float4*>(wr + ii));
+          part = fmaf(av.x, wv.x, fmaf(av.y, wv.y, fmaf(av.z, wv.z, fmaf(av.w, wv.w, part))));
+        }
+        if (P.m[t]) part *= __ldg(P.m[t] + hs * H + ws);
+        acc += part;
+      }
+      P.d[idx] = fmaxf(acc * __ldg(P.s2 + o) + __ldg(P.b2 + o), 0.f);
+    }
+  }
+  stamp(P, 2);
+  grid_sync(P, 1);
+  // ---- 3: 1x1 convolution (+ BN) + shortcut + ReLU
+  gemm_tasks(P.d, w, ident, P.W3, HWo, cout, w, 0, tsm, [&](int m, int n, float v) {
+    const int64_t o = (int64_t)m * cout + n;
+    const float sc = P.Wd ? P.y[o] : __ldg(P.x + o);
+    P.y[o] = fmaxf(v * __ldg(P.s3 + n) + __ldg(P.b3 + n) + sc, 0.f);
+  });
+  stamp(P, 3);
+  // ---- exit: the last CTA resets the barrier counters for the next launch
+  __syncthreads();
+  __shared__ int last;
+  if (tid == 0) {
+    __threadfence();
+    last = atomicAdd(&P.ctrl[4], 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last && tid == 0) {
+    __threadfence();
+    P.ctrl[0] = P.ctrl[1] = P.ctrl[4] = 0u;
+    __threadfence();
+  }
+}
+
+}  // namespace rx
+
+cudaError_t resnext_launch(const RxParams& prm, int grid, cudaStream_t s) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(RX_THREADS);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;   // the grid barriers need every CTA co-resident
+  at[0].val.cooperative = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  const int cg = prm.w / prm.G;
+  void (*fn)(RxParams) = cg == 4 ? rx::resnext_kernel<4> : cg == 8 ? rx::resnext_kernel<8>
+                       : cg == 16 ? rx::resnext_kernel<16> : cg == 32 ? rx::resnext_kernel<32> : rx::resnext_kernel<0>;
+  return cudaLaunchKernelEx(&cfg, fn, prm);
+}
+
+}  // namespace souffle

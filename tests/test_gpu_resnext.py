@@ -1,5 +1,5 @@
 """GPU parity of the ResNeXt Bottleneck blocks (Table 2, ResNeXt-101 64 x 4d; SURVEY
-§8(f) NEXT-3) on the generic fused-subprogram executor against the fp64 oracle: fp32 TEs, max_i |g_i -
+§8(f) NEXT-3) on the pattern kernel and on the generic fused-subprogram executor against the fp64 oracle: fp32 TEs, max_i |g_i -
 o_i| / max(|o_i|, rms(o)) <= 1e-4.  The grouped 3x3 convolution runs as 9 batched-matmul TEs over the
 64 groups whose rolled + masked A operands are gathered through the index maps (stencil gathers)."""
 import numpy as np
@@ -36,10 +36,20 @@ def _case(cfg, flags=0):
 
 
 @pytest.mark.parametrize("i", range(8), ids=[c["name"] for c in synth.RESNEXT_CONFIGS])
-def test_resnext_block_generic(i, record_err):
+def test_resnext_block_pattern(i, record_err):
+    """The ResNeXt pattern kernel (kernels/resnext.cu): one persistent launch, two grid barriers."""
     cfg = synth.RESNEXT_CONFIGS[i]
     out, ref, plan = _case(cfg)
-    record_err(rel_err(out, ref), 1e-4, block=cfg["name"], launches=plan.exec_info()["launches"])
+    assert "pattern resnext:" in plan.describe() and plan.exec_info()["launches"] == 1
+    record_err(rel_err(out, ref), 1e-4, block=cfg["name"], path="pattern")
+
+
+@pytest.mark.parametrize("i", range(8), ids=[c["name"] for c in synth.RESNEXT_CONFIGS])
+def test_resnext_block_generic(i, record_err):
+    cfg = synth.RESNEXT_CONFIGS[i]
+    out, ref, plan = _case(cfg, L.FLAG_NO_PATTERN)
+    assert "pattern resnext: not used" in plan.describe()
+    record_err(rel_err(out, ref), 1e-4, block=cfg["name"], launches=plan.exec_info()["launches"], path="generic")
 
 
 @pytest.mark.parametrize("flags", [L.FLAG_UNFUSED, L.FLAG_NO_GLOBAL_SYNC])
