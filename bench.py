@@ -519,6 +519,32 @@ def main():
                                         "modules": mb_rows,
                                         "geomean_speedup_vs_unfused": float(np.exp(np.mean([np.log(r["speedup"]) for r in mb_rows]))),
                                         "kernel": "kernels/mbconv.cu (one persistent launch, Fig. 5(c))"}
+        # ResNeXt-101 64x4d Bottleneck blocks R0-R7 (Table 2): the pattern kernel (one persistent
+        # launch) against the unfused one-kernel-per-TE path; the 33 blocks of the network (layers
+        # [3, 4, 23, 3]: each stage's first block + its repeated block) summed from the per-block times
+        progress("ResNeXt blocks")
+        rx_rows = []
+        for cfg in _synth.RESNEXT_CONFIGS:
+            ps_ = {**_synth.resnext_params(cfg), **_synth.resnext_masks(cfg)}
+            g_, nm_, gx_, gy_ = M.resnext(cfg)
+            row = {"block": cfg["name"], "cin": cfg["cin"], "width": cfg["width"], "cout": cfg["cout"],
+                   "stride": cfg["stride"], "hw": cfg["hw"]}
+            for key, fl in (("pattern_us", 0), ("unfused_us", L.FLAG_UNFUSED)):
+                pl_ = g_.partition(L.device_query(local), fl)
+                ss_ = _session(g_, pl_, {nm_[k]: v for k, v in ps_.items()} | {gx_: _synth.resnext_input(cfg)}, [gy_],
+                               device=f"cuda:{local}")
+                row[key] = statistics.median(time_steps(ss_, 20, 3, flush, stream)) * 1e3
+                del ss_, pl_
+            row["speedup"] = row["unfused_us"] / row["pattern_us"]
+            rx_rows.append(row)
+        reps = [1, 2, 1, 3, 1, 22, 1, 2]   # R0 + 2 R1 | R2 + 3 R3 | R4 + 22 R5 | R6 + 2 R7
+        extra["resnext"] = {"workload": "ResNeXt-101 64x4d Bottleneck blocks R0-R7 (fp32, batch 1)",
+                            "blocks": rx_rows,
+                            "geomean_speedup_vs_unfused": float(np.exp(np.mean([np.log(r["speedup"]) for r in rx_rows]))),
+                            "network_33_blocks_us": float(sum(n * r["pattern_us"] for n, r in zip(reps, rx_rows))),
+                            "network_note": "sum of the 33 Bottleneck blocks only (no stem, pooling or classifier)",
+                            "paper_a100_ms": 4.43,
+                            "kernel": "kernels/resnext.cu (one persistent launch, 2 grid barriers)"}
         # Swin-B runs in a child process (fresh CUDA context) with a time limit: a launch that trips a
         # kernel watchdog must not take the whole bench line with it
         progress("Swin-B (child process)")
