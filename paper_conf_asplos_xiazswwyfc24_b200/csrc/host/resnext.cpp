@@ -148,7 +148,13 @@ void resnext_match(const Graph& g, const Analysis& an, const souffle_device_desc
   rp.o_ctrl = o; o = al(o + 256, 256);
   rp.o_a = o; o = al(o + 4 * HW * w, 256);
   rp.o_d = o; o = al(o + 4 * Ho * Ho * w, 256);
+  rp.o_acc1 = o; o = al(o + 4 * HW * w, 256);
+  rp.o_acc2 = o; o = al(o + 4 * Ho * Ho * cout, 256);
+  rp.o_acc3 = o; o = al(o + 4 * Ho * Ho * cout, 256);
+  rp.o_cnt = o; o = al(o + 4 * 3 * RX_MAX_TILES, 256);
   rp.total = al(o, 4096);
+  if ((HW + 63) / 64 * ((w + 63) / 64) > RX_MAX_TILES || (Ho * Ho + 63) / 64 * ((cout + 63) / 64) > RX_MAX_TILES)
+    return no("too many 64 x 64 GEMM tiles for the split-K counters");
   rp.on = true;
 }
 
@@ -182,6 +188,10 @@ souffle_status resnext_run(Plan& p, void* ws, void* stream) {
   prm.a = (float*)(base + rp.o_a);
   prm.d = (float*)(base + rp.o_d);
   prm.ctrl = (unsigned*)(base + rp.o_ctrl);
+  prm.acc1 = (float*)(base + rp.o_acc1);
+  prm.acc2 = (float*)(base + rp.o_acc2);
+  prm.acc3 = (float*)(base + rp.o_acc3);
+  prm.cnt = (unsigned*)(base + rp.o_cnt);
   if (std::getenv("SOUFFLE_RX_PROF")) prm.prof = (unsigned long long*)(base + rp.o_ctrl + 64);   // 4 stamps
   prm.H = rp.H; prm.cin = rp.cin; prm.w = rp.w; prm.G = rp.G; prm.stride = rp.stride; prm.cout = rp.cout;
   cudaError_t e = resnext_launch(prm, rp.grid, (cudaStream_t)stream);

@@ -47,8 +47,8 @@ __device__ __forceinline__ float4 ld_ca4(const float* p) {
 // C[m0.., n0..] (BM x BN) = sum_k A(arow(m), k) B[n][k]; epi(m, n, v) for the in-range outputs.  256
 // threads, (BM/16) x (BN/16) outputs each; K in slabs of 16 staged k-major in shared memory.
 template <int BM, int BN, class Row, class Epi>
-__device__ __forceinline__ void tile(const float* A, int lda, Row arow, const float* B, int M, int N, int K, int m0,
-                                     int n0, float* sm, Epi epi) {
+__device__ __forceinline__ void tile(const float* A, int lda, Row arow, const float* B, int M, int N, int K, int kbeg,
+                                     int kend, int m0, int n0, float* sm, Epi epi) {
   constexpr int RM = BM / 16, RN = BN / 16;
   float(*As)[BM + 1] = reinterpret_cast<float(*)[BM + 1]>(sm);
   float(*Bs)[BN + 1] = reinterpret_cast<float(*)[BN + 1]>(sm + 16 * (BM + 1));
@@ -58,17 +58,17 @@ __device__ __forceinline__ void tile(const float* A, int lda, Row arow, const fl
   for (int i = 0; i < RM; ++i)
 #pragma unroll
     for (int j = 0; j < RN; ++j) c[i][j] = 0.f;
-  for (int k0 = 0; k0 < K; k0 += 16) {
+  for (int k0 = kbeg; k0 < kend; k0 += 16) {
     __syncthreads();
 #pragma unroll
     for (int q = 0; q < (BM * 16) / RX_THREADS; ++q) {
       const int e = tid + q * RX_THREADS, kk = e & 15, r = e >> 4, k = k0 + kk;
-      As[kk][r] = (m0 + r < M && k < K) ? __ldcg(A + (int64_t)arow(m0 + r) * lda + k) : 0.f;
+      As[kk][r] = (m0 + r < M && k < kend) ? __ldcg(A + (int64_t)arow(m0 + r) * lda + k) : 0.f;
     }
 #pragma unroll
     for (int q = 0; q < (BN * 16) / RX_THREADS; ++q) {
       const int e = tid + q * RX_THREADS, kk = e & 15, r = e >> 4, k = k0 + kk;
-      Bs[kk][r] = (n0 + r < N && k < K) ? __ldg(B + (int64_t)(n0 + r) * K + k) : 0.f;
+      Bs[kk][r] = (n0 + r < N && k < kend) ? __ldg(B + (int64_t)(n0 + r) * K + k) : 0.f;
     }
     __syncthreads();
 #pragma unroll
@@ -93,18 +93,52 @@ __device__ __forceinline__ void tile(const float* A, int lda, Row arow, const fl
     }
 }
 
-// the tiles of one GEMM, task t0.. of a shared task space: 64 x 64 tiles when they fill half the grid,
-// else 32 x 32.  Returns the number of tasks it has.
+// the tiles of one GEMM, task t0.. of a shared task space: 64 x 64 tiles when they fill half the grid.
+// Otherwise (the small-M blocks: 196 or 49 pixels) split K over 64 x 64 tiles when an fp32 accumulator
+// is given -- 4 x 4 outputs per thread instead of the 2 x 2 of 32 x 32 tiles, half the shared-memory
+// traffic per FMA -- the splits add into acc (atomics) and the last split of a tile (per-tile arrival
+// counter) runs the epilogue and clears acc / its counter for the next launch; else 32 x 32 tiles.
+// Returns the number of tasks it has.
 template <class Row, class Epi>
 __device__ __forceinline__ int gemm_tasks(const float* A, int lda, Row arow, const float* B, int M, int N, int K,
-                                          int t0, float* sm, Epi epi) {
-  const int t64 = ((M + 63) / 64) * ((N + 63) / 64);
+                                          int t0, float* sm, Epi epi, float* acc = nullptr, unsigned* cnt = nullptr) {
+  const int tn64 = (N + 63) / 64, t64 = ((M + 63) / 64) * tn64;
   const bool big = 2 * t64 >= (int)gridDim.x;
+  if (!big && acc && K >= 256) {
+    const int sp = max(1, min((int)gridDim.x / t64, K / 128));
+    const int kper = ((K + sp - 1) / sp + 15) / 16 * 16, nt = t64 * sp;
+    __shared__ int last;
+    for (int t = (int)blockIdx.x - t0; t < nt; t += gridDim.x) {
+      if (t < 0) continue;
+      const int tile_id = t / sp, ks = (t % sp) * kper;
+      const int m0 = (tile_id / tn64) * 64, n0 = (tile_id % tn64) * 64;
+      tile<64, 64>(A, lda, arow, B, M, N, K, ks, min(K, ks + kper), m0, n0, sm,
+                   [&](int m, int n, float v) { atomicAdd(acc + (int64_t)m * N + n, v); });
+      __threadfence();
+      __syncthreads();
+      if (threadIdx.x == 0) last = atomicAdd(cnt + tile_id, 1u) == (unsigned)sp - 1;
+      __syncthreads();
+      if (last) {
+        __threadfence();
+        for (int e = threadIdx.x; e < 64 * 64; e += RX_THREADS) {
+          const int m = m0 + e / 64, n = n0 + e % 64;
+          if (m < M && n < N) {
+            float* pa = acc + (int64_t)m * N + n;
+            const float v = __ldcg(pa);
+            *pa = 0.f;
+            epi(m, n, v);
+          }
+        }
+        if (threadIdx.x == 0) cnt[tile_id] = 0u;
+      }
+    }
+    return nt;
+  }
   const int bm = big ? 64 : 32, tn = (N + bm - 1) / bm, nt = ((M + bm - 1) / bm) * tn;
   for (int t = (int)blockIdx.x - t0; t < nt; t += gridDim.x) {
     if (t < 0) continue;
-    if (big) tile<64, 64>(A, lda, arow, B, M, N, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
-    else tile<32, 32>(A, lda, arow, B, M, N, K, (t / tn) * 32, (t % tn) * 32, sm, epi);
+    if (big) tile<64, 64>(A, lda, arow, B, M, N, K, 0, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
+    else tile<32, 32>(A, lda, arow, B, M, N, K, 0, K, (t / tn) * 32, (t % tn) * 32, sm, epi);
   }
   return nt;
 }
@@ -123,12 +157,12 @@ __global__ void __launch_bounds__(RX_THREADS, 1) resnext_kernel(const __grid_con
   // task numbering so the two GEMMs share the grid)
   const int n1 = gemm_tasks(P.x, cin, ident, P.W1, HW, w, cin, 0, tsm, [&](int m, int n, float v) {
     P.a[(int64_t)m * w + n] = fmaxf(v * __ldg(P.s1 + n) + __ldg(P.b1 + n), 0.f);
-  });
+  }, P.acc1, P.cnt);
   if (P.Wd) {
     auto srow = [&](int m) { return (m / Ho) * s * H + (m % Ho) * s; };   // output pixel -> input row
     gemm_tasks(P.x, cin, srow, P.Wd, HWo, cout, cin, n1 % (int)gridDim.x, tsm, [&](int m, int n, float v) {
       P.y[(int64_t)m * cout + n] = v * __ldg(P.sd + n) + __ldg(P.bd + n);
-    });
+    }, P.acc2, P.cnt + RX_MAX_TILES);
   }
   stamp(P, 1);
   grid_sync(P, 0);
@@ -167,7 +201,7 @@ __global__ void __launch_bounds__(RX_THREADS, 1) resnext_kernel(const __grid_con
     const int64_t o = (int64_t)m * cout + n;
     const float sc = P.Wd ? P.y[o] : __ldg(P.x + o);
     P.y[o] = fmaxf(v * __ldg(P.s3 + n) + __ldg(P.b3 + n) + sc, 0.f);
-  });
+  }, P.acc3, P.cnt + 2 * RX_MAX_TILES);
   stamp(P, 3);
   // ---- exit: the last CTA resets the barrier counters for the next launch
   __syncthreads();

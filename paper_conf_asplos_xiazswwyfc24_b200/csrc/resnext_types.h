@@ -15,7 +15,7 @@
 
 namespace souffle {
 
-enum { RX_THREADS = 256, RX_TAPS = 9 };
+enum { RX_THREADS = 256, RX_TAPS = 9, RX_MAX_TILES = 1024 };
 
 struct RxParams {
   const float* x;                 // [H*H][cin]
@@ -36,6 +36,10 @@ struct RxParams {
   float* a;                       // workspace [H*H][w]
   float* d;                       // workspace [Ho*Ho][w]
   unsigned* ctrl;                 // [0..1] grid barriers, [4] exit counter
+  float* acc1;                    // split-K fp32 accumulators (zero between launches) of the 1x1 GEMM,
+  float* acc2;                    // the projection and the second 1x1 GEMM
+  float* acc3;
+  unsigned* cnt;                  // [3][RX_MAX_TILES] per-tile split arrival counters (zero between launches)
   unsigned long long* prof;       // debug (SOUFFLE_RX_PROF): %globaltimer of CTA 0 at the phase boundaries [4]
   int32_t H, cin, w, G, stride, cout, pad0, pad1;
 };
