@@ -13,5 +13,7 @@ timeout 1500 python bench.py > gpurun_out/r02_bench.json 2> gpurun_out/r02_bench
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/r02_launches.csv python bench.py --steps 3 --warmup 3 --no-cpu-baseline --no-v0 --no-models > gpurun_out/r02_ncu_launch.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:bert_kernel -s 1 -c 1 -o gpurun_out/r02_prof_bert python tools/run_once.py bert_base 0 0 2 > gpurun_out/r02_ncu_full.log 2>&1
 timeout 300 python tools/profile_bert.py 12 > gpurun_out/r02_timeline.txt 2>&1
+timeout 600 ncu --set full --clock-control none -k regex:mmoe_cluster_kernel -s 3 -c 1 -o gpurun_out/r02_prof_mmoe python tools/run_model_once.py mmoe 6 > gpurun_out/r02_ncu_mmoe.log 2>&1
+timeout 600 python tools/profile_resnext.py > gpurun_out/r02_resnext_phases.txt 2>&1
 for b in 1 8 64; do timeout 300 python tools/swin_trace.py $b > gpurun_out/r02_swin_trace_b$b.txt 2>&1; done
 echo done
