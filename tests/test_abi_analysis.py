@@ -343,3 +343,18 @@ def test_mmoe_kernel_variant_policy(monkeypatch):
     assert "in one CTA" in describe(**big)
     monkeypatch.setenv("SOUFFLE_MMOE_SINGLE", "1")
     assert "in one CTA" in describe()
+
+
+def test_resnext_pattern_matches_and_skips_generic_lowering():
+    """The ResNeXt Bottleneck programs R0-R7 are matched by the ResNeXt pattern (one persistent launch,
+    two grid barriers) on the host, the generic lowering skipped; ablation flags select the generic
+    executor (whose partition splits the 9 grouped taps over several subprograms)."""
+    for cfg in synth.RESNEXT_CONFIGS:
+        g = M.resnext(cfg)[0]
+        plan = g.partition(L.device_b200())
+        d = plan.describe()
+        assert "pattern resnext: " in d and "pattern resnext: not used" not in d, d[:400]
+        assert plan.exec_info() == {"launches": 1, "stages": 3, "barriers": 2}
+        assert ("projection shortcut" in d) == synth.resnext_projection(cfg)
+    g = M.resnext(synth.RESNEXT_CONFIGS[5])[0]
+    assert "pattern resnext: not used" in g.partition(L.device_b200(), flags=L.FLAG_UNFUSED).describe()
