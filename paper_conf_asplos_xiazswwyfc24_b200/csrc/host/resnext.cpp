@@ -139,6 +139,7 @@ void resnext_match(const Graph& g, const Analysis& an, const souffle_device_desc
   }
   y = c.ew(SOUFFLE_EW_RELU, {c.ew(SOUFFLE_EW_ADD, {y, sc})});
   if (!c.ok || c.i != N.size()) return no("not a ResNeXt block");
+  if (cin % 16 || w % 16 || cout % 16) return no("channel counts must be multiples of 16 (vector GEMM slabs)");
   if (g.outputs.size() != 1 || g.outputs[0] != y) return no("the only output must be the block output");
   const int sms = dev.num_sms > 0 ? dev.num_sms : 148;
   rp.y = y;

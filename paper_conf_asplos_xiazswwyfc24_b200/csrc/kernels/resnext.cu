@@ -93,6 +93,68 @@ __device__ __forceinline__ void tile(const float* A, int lda, Row arow, const fl
     }
 }
 
+// 64 x 64 tile, 4 x 4 outputs per thread, K in slabs of 16: each thread loads one float4 of A and of B
+// per slab (the next slab's pair is fetched into registers while the current one is multiplied) and
+// stores it transposed (k-major rows of 68 floats: 16-byte aligned, conflict-free stores), and every
+// k step reads its 4 A and 4 B values as two 128-bit shared loads (2 loads per 16 FMA).  Requires
+// lda, K, kbeg, kend multiples of 4 (the matcher checks 16).  A through L1 (ld.global.ca: the input x,
+// or d written before the last grid barrier, never written again in the launch).
+template <class Row, class Epi>
+__device__ __forceinline__ void tile64(const float* A, int lda, Row arow, const float* B, int M, int N, int K, int kbeg,
+                                       int kend, int m0, int n0, float* sm, Epi epi) {
+  constexpr int LD = 68;
+  float(*As)[LD] = reinterpret_cast<float(*)[LD]>(sm);
+  float(*Bs)[LD] = reinterpret_cast<float(*)[LD]>(sm + 16 * LD);
+  const int tid = threadIdx.x, ty = tid >> 4, tx = tid & 15;
+  const int lr = tid & 63, lq = tid >> 6;   // loader: row lr of the tile, k quad lq of the slab
+  const bool arow_ok = m0 + lr < M, brow_ok = n0 + lr < N;
+  const float* ap = A + (int64_t)(arow_ok ? arow(m0 + lr) : 0) * lda + 4 * lq;
+  const float* bp = B + (int64_t)(brow_ok ? n0 + lr : 0) * K + 4 * lq;
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  auto lda4 = [&](int k0) {
+    if (!arow_ok || k0 + 4 * lq >= kend) return z4;
+    float4 v;
+    asm volatile("ld.global.ca.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(ap + k0));
+    return v;
+  };
+  auto ldb4 = [&](int k0) {
+    return (!brow_ok || k0 + 4 * lq >= kend) ? z4 : __ldg(reinterpret_cast<const float4*>(bp + k0));
+  };
+  float c[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) c[i][j] = 0.f;
+  float4 an = lda4(kbeg), bn = ldb4(kbeg);
+  for (int k0 = kbeg; k0 < kend; k0 += 16) {
+    __syncthreads();
+    As[4 * lq + 0][lr] = an.x; As[4 * lq + 1][lr] = an.y; As[4 * lq + 2][lr] = an.z; As[4 * lq + 3][lr] = an.w;
+    Bs[4 * lq + 0][lr] = bn.x; Bs[4 * lq + 1][lr] = bn.y; Bs[4 * lq + 2][lr] = bn.z; Bs[4 * lq + 3][lr] = bn.w;
+    __syncthreads();
+    if (k0 + 16 < kend) {
+      an = lda4(k0 + 16);
+      bn = ldb4(k0 + 16);
+    }
+#pragma unroll
+    for (int kk = 0; kk < 16; ++kk) {
+      const float4 a4 = *reinterpret_cast<const float4*>(&As[kk][4 * ty]);
+      const float4 b4 = *reinterpret_cast<const float4*>(&Bs[kk][4 * tx]);
+      const float av[4] = {a4.x, a4.y, a4.z, a4.w}, bv[4] = {b4.x, b4.y, b4.z, b4.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) c[i][j] = fmaf(av[i], bv[j], c[i][j]);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int m = m0 + 4 * ty + i, n = n0 + 4 * tx + j;
+      if (m < M && n < N) epi(m, n, c[i][j]);
+    }
+}
+
 // the tiles of one GEMM, task t0.. of a shared task space: 64 x 64 tiles when they fill half the grid.
 // Otherwise (the small-M blocks: 196 or 49 pixels) split K over 64 x 64 tiles when an fp32 accumulator
 // is given -- 4 x 4 outputs per thread instead of the 2 x 2 of 32 x 32 tiles, half the shared-memory
@@ -112,7 +174,7 @@ __device__ __forceinline__ int gemm_tasks(const float* A, int lda, Row arow, con
       if (t < 0) continue;
       const int tile_id = t / sp, ks = (t % sp) * kper;
       const int m0 = (tile_id / tn64) * 64, n0 = (tile_id % tn64) * 64;
-      tile<64, 64>(A, lda, arow, B, M, N, K, ks, min(K, ks + kper), m0, n0, sm,
+      tile64(A, lda, arow, B, M, N, K, ks, min(K, ks + kper), m0, n0, sm,
                    [&](int m, int n, float v) { atomicAdd(acc + (int64_t)m * N + n, v); });
       __threadfence();
       __syncthreads();
@@ -137,7 +199,7 @@ __device__ __forceinline__ int gemm_tasks(const float* A, int lda, Row arow, con
   const int bm = big ? 64 : 32, tn = (N + bm - 1) / bm, nt = ((M + bm - 1) / bm) * tn;
   for (int t = (int)blockIdx.x - t0; t < nt; t += gridDim.x) {
     if (t < 0) continue;
-    if (big) tile<64, 64>(A, lda, arow, B, M, N, K, 0, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
+    if (big) tile64(A, lda, arow, B, M, N, K, 0, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
     else tile<32, 32>(A, lda, arow, B, M, N, K, 0, K, (t / tn) * 32, (t % tn) * 32, sm, epi);
   }
   return nt;
@@ -145,7 +207,7 @@ __device__ __forceinline__ int gemm_tasks(const float* A, int lda, Row arow, con
 
 template <int CG>   // channels per group (0: any, loops not unrolled)
 __global__ void __launch_bounds__(RX_THREADS, 1) resnext_kernel(const __grid_constant__ RxParams P) {
-  __shared__ float tsm[2 * 16 * 65];   // GEMM operand slabs
+  __shared__ __align__(16) float tsm[2 * 16 * 68];   // GEMM operand slabs
   const int tid = threadIdx.x;
   const int H = P.H, w = P.w, s = P.stride, cout = P.cout, cin = P.cin;
   const int HW = H * H, Ho = H / s, HWo = Ho * Ho;
