@@ -9,6 +9,7 @@
 //   sw_row_kernel   LayerNorm of rows gathered through the block's quasi-affine index maps
 //   sw_im2col_kernel, sw_head_kernel   patch embedding gather; final LN + mean pool + classifier
 #include <cuda.h>
+#include <cstdlib>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -819,53 +820,72 @@ __global__ void __launch_bounds__(SW_ATTN_THREADS) sw_attn_kernel(const __grid_c
 // One warp per output row; lane l holds float4 column groups l, l + 32, ... (NV groups).  The
 // statistics are merged pairwise (Chan) from exactly centred per-lane values: a constant row gives
 // exactly beta, an offset row keeps its noise (no E[x^2] - E[x]^2 cancellation).
-template <int NV>
+// RPW rows per warp (narrow rows: C = 128 or 256): every row's gather-index loads are issued, then every
+// row's data loads, so a warp keeps RPW x NV float4 requests in flight instead of NV (the narrow stages
+// were bound by the bytes in flight per SM, not by HBM).
+template <int NV, int RPW>
 __global__ void __launch_bounds__(SW_ROW_THREADS) sw_row_kernel(const SwRow R) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   pdl_trigger();
   pdl_wait();
   trace_stamp(R.trace, R.op);
-  const int r = blockIdx.x * (SW_ROW_THREADS / 32) + warp;
-  if (r >= R.rows) return;
+  const int rbase = (blockIdx.x * (SW_ROW_THREADS / 32) + warp) * RPW;
+  if (rbase >= R.rows) return;
   const int cin = R.cols / R.nsrc;
-  float4 v[NV];
+  int tok[RPW][NV];
 #pragma unroll
-  for (int k = 0; k < NV; ++k) {
-    const int e = 4 * (lane + 32 * k);
-    const int s = e / cin, o = e - s * cin;
-    const int tok = R.src ? __ldg(R.src + (int64_t)r * R.nsrc + s) : r;
-    v[k] = __ldg(reinterpret_cast<const float4*>(R.x + (int64_t)tok * cin + o));
-  }
-  float m = 0.f;
+  for (int q = 0; q < RPW; ++q)
 #pragma unroll
-  for (int k = 0; k < NV; ++k) m += (v[k].x + v[k].y) + (v[k].z + v[k].w);
-  m *= 1.f / (float)(4 * NV);
-  float M2 = 0.f;
+    for (int k = 0; k < NV; ++k) {
+      const int r = min(rbase + q, R.rows - 1);
+      const int e = 4 * (lane + 32 * k);
+      const int s = e / cin;
+      tok[q][k] = R.src ? __ldg(R.src + (int64_t)r * R.nsrc + s) : r;
+    }
+  float4 v[RPW][NV];
 #pragma unroll
-  for (int k = 0; k < NV; ++k) {
-    const float a = v[k].x - m, b = v[k].y - m, c = v[k].z - m, d = v[k].w - m;
-    M2 += (a * a + b * b) + (c * c + d * d);
-  }
-  float n = (float)(4 * NV);
+  for (int q = 0; q < RPW; ++q)
 #pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const float mb = __shfl_xor_sync(0xffffffffu, m, o), Mb = __shfl_xor_sync(0xffffffffu, M2, o);
-    const float dl = mb - m;
-    M2 = (M2 + Mb) + dl * dl * (0.5f * n);
-    m = (m + mb) * 0.5f;
-    n *= 2.f;
-  }
-  const float rs = rsqrtf(M2 / (float)R.cols + R.eps);
+    for (int k = 0; k < NV; ++k) {
+      const int e = 4 * (lane + 32 * k);
+      const int s = e / cin, o = e - s * cin;
+      v[q][k] = __ldg(reinterpret_cast<const float4*>(R.x + (int64_t)tok[q][k] * cin + o));
+    }
 #pragma unroll
-  for (int k = 0; k < NV; ++k) {
-    const int e = 4 * (lane + 32 * k);
-    const float4 gm = __ldg(reinterpret_cast<const float4*>(R.gamma + e));
-    const float4 bt = __ldg(reinterpret_cast<const float4*>(R.beta + e));
-    const float4 y = make_float4((v[k].x - m) * rs * gm.x + bt.x, (v[k].y - m) * rs * gm.y + bt.y,
-                                 (v[k].z - m) * rs * gm.z + bt.z, (v[k].w - m) * rs * gm.w + bt.w);
-    if (R.out_b)
-      *reinterpret_cast<uint2*>(R.out_b + (int64_t)r * R.cols + e) = make_uint2(pack_bf16(y.x, y.y), pack_bf16(y.z, y.w));
-    if (R.out_f) *reinterpret_cast<float4*>(R.out_f + (int64_t)r * R.cols + e) = y;
+  for (int q = 0; q < RPW; ++q) {
+    const int r = rbase + q;
+    float m = 0.f;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) m += (v[q][k].x + v[q][k].y) + (v[q][k].z + v[q][k].w);
+    m *= 1.f / (float)(4 * NV);
+    float M2 = 0.f;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+      const float a = v[q][k].x - m, b = v[q][k].y - m, c = v[q][k].z - m, d = v[q][k].w - m;
+      M2 += (a * a + b * b) + (c * c + d * d);
+    }
+    float n = (float)(4 * NV);
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const float mb = __shfl_xor_sync(0xffffffffu, m, o), Mb = __shfl_xor_sync(0xffffffffu, M2, o);
+      const float dl = mb - m;
+      M2 = (M2 + Mb) + dl * dl * (0.5f * n);
+      m = (m + mb) * 0.5f;
+      n *= 2.f;
+    }
+    if (r >= R.rows) continue;
+    const float rs = rsqrtf(M2 / (float)R.cols + R.eps);
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+      const int e = 4 * (lane + 32 * k);
+      const float4 gm = __ldg(reinterpret_cast<const float4*>(R.gamma + e));
+      const float4 bt = __ldg(reinterpret_cast<const float4*>(R.beta + e));
+      const float4 y = make_float4((v[q][k].x - m) * rs * gm.x + bt.x, (v[q][k].y - m) * rs * gm.y + bt.y,
+                                   (v[q][k].z - m) * rs * gm.z + bt.z, (v[q][k].w - m) * rs * gm.w + bt.w);
+      if (R.out_b)
+        *reinterpret_cast<uint2*>(R.out_b + (int64_t)r * R.cols + e) = make_uint2(pack_bf16(y.x, y.y), pack_bf16(y.z, y.w));
+      if (R.out_f) *reinterpret_cast<float4*>(R.out_f + (int64_t)r * R.cols + e) = y;
+    }
   }
 }
 
@@ -1115,13 +1135,19 @@ cudaError_t sw_launch_attn(const void* tq, const void* tk, const void* tv, const
 }
 
 cudaError_t sw_launch_row(const SwRow& r, cudaStream_t s) {
-  const dim3 grid((r.rows + 7) / 8), blk(SW_ROW_THREADS);
+  // rows per warp: 4 for C = 128, 2 for C = 256 (SOUFFLE_SWIN_LN_RPW1=1: one row per warp, studies)
+  static const bool one = std::getenv("SOUFFLE_SWIN_LN_RPW1") != nullptr;
+  int rpw = one ? 1 : r.cols == 128 ? 4 : r.cols == 256 ? 2 : 1;
+  if ((r.rows + 8 * rpw - 1) / (8 * rpw) < 2 * 148) rpw = 1;   // small batches: keep the CTAs (b1: -1 %)
+  const dim3 grid((r.rows + 8 * rpw - 1) / (8 * rpw)), blk(SW_ROW_THREADS);
   switch (r.cols / 128) {
-    case 1: return launch_pdl(swin::sw_row_kernel<1>, grid, blk, 0, s, r);
-    case 2: return launch_pdl(swin::sw_row_kernel<2>, grid, blk, 0, s, r);
-    case 4: return launch_pdl(swin::sw_row_kernel<4>, grid, blk, 0, s, r);
-    case 8: return launch_pdl(swin::sw_row_kernel<8>, grid, blk, 0, s, r);
-    case 16: return launch_pdl(swin::sw_row_kernel<16>, grid, blk, 0, s, r);
+    case 1: return rpw == 4 ? launch_pdl(swin::sw_row_kernel<1, 4>, grid, blk, 0, s, r)
+                            : launch_pdl(swin::sw_row_kernel<1, 1>, grid, blk, 0, s, r);
+    case 2: return rpw == 2 ? launch_pdl(swin::sw_row_kernel<2, 2>, grid, blk, 0, s, r)
+                            : launch_pdl(swin::sw_row_kernel<2, 1>, grid, blk, 0, s, r);
+    case 4: return launch_pdl(swin::sw_row_kernel<4, 1>, grid, blk, 0, s, r);
+    case 8: return launch_pdl(swin::sw_row_kernel<8, 1>, grid, blk, 0, s, r);
+    case 16: return launch_pdl(swin::sw_row_kernel<16, 1>, grid, blk, 0, s, r);
     default: return cudaErrorInvalidValue;
   }
 }
