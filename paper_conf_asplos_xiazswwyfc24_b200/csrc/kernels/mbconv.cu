@@ -107,6 +107,69 @@ __device__ __forceinline__ void tile(const float* A, int lda, const float* ascal
     }
 }
 
+// 64 x 64 tile with 4 x 4 outputs per thread: one float4 of A and of B per thread and 16-deep slab,
+// the next slab's pair fetched into registers while the current one is multiplied, transposed into
+// 16-byte-aligned k-major rows (68 floats) and read back as two 128-bit shared loads per 16 FMA.  A
+// through L1 (written before the last grid barrier, never again in the launch), scaled by ascale[k]
+// when given.  Needs lda and K multiples of 4 (every MBConv channel count is).
+template <class Epi>
+__device__ __forceinline__ void tile64(const float* A, int lda, const float* ascale, const float* B, int ldb, int M,
+                                       int N, int kbeg, int kend, int m0, int n0, float* sm, Epi epi) {
+  constexpr int LD = 68;
+  float(*As)[LD] = reinterpret_cast<float(*)[LD]>(sm);
+  float(*Bs)[LD] = reinterpret_cast<float(*)[LD]>(sm + 16 * LD);
+  const int tid = threadIdx.x, ty = tid >> 4, tx = tid & 15;
+  const int lr = tid & 63, lq = tid >> 6;
+  const bool aok = m0 + lr < M, bok = n0 + lr < N;
+  const float* ap = A + (int64_t)(aok ? m0 + lr : 0) * lda + 4 * lq;
+  const float* bp = B + (int64_t)(bok ? n0 + lr : 0) * ldb + 4 * lq;
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  auto lda4 = [&](int k0) {
+    if (!aok || k0 + 4 * lq >= kend) return z4;
+    float4 v;
+    asm volatile("ld.global.ca.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(ap + k0));
+    if (ascale) {
+      const int k = k0 + 4 * lq;
+      v.x *= ascale[k]; v.y *= ascale[k + 1]; v.z *= ascale[k + 2]; v.w *= ascale[k + 3];
+    }
+    return v;
+  };
+  auto ldb4 = [&](int k0) { return (!bok || k0 + 4 * lq >= kend) ? z4 : __ldg(reinterpret_cast<const float4*>(bp + k0)); };
+  float c[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) c[i][j] = 0.f;
+  float4 an = lda4(kbeg), bn = ldb4(kbeg);
+  for (int k0 = kbeg; k0 < kend; k0 += 16) {
+    __syncthreads();
+    As[4 * lq + 0][lr] = an.x; As[4 * lq + 1][lr] = an.y; As[4 * lq + 2][lr] = an.z; As[4 * lq + 3][lr] = an.w;
+    Bs[4 * lq + 0][lr] = bn.x; Bs[4 * lq + 1][lr] = bn.y; Bs[4 * lq + 2][lr] = bn.z; Bs[4 * lq + 3][lr] = bn.w;
+    __syncthreads();
+    if (k0 + 16 < kend) {
+      an = lda4(k0 + 16);
+      bn = ldb4(k0 + 16);
+    }
+#pragma unroll
+    for (int kk = 0; kk < 16; ++kk) {
+      const float4 a4 = *reinterpret_cast<const float4*>(&As[kk][4 * ty]);
+      const float4 b4 = *reinterpret_cast<const float4*>(&Bs[kk][4 * tx]);
+      const float av[4] = {a4.x, a4.y, a4.z, a4.w}, bv[4] = {b4.x, b4.y, b4.z, b4.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) c[i][j] = fmaf(av[i], bv[j], c[i][j]);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int m = m0 + 4 * ty + i, n = n0 + 4 * tx + j;
+      if (m < M && n < N) epi(m, n, c[i][j]);
+    }
+}
+
 // a GEMM phase over output tiles: 64 x 64 tiles when they fill half the grid, else 32 x 32
 template <class Epi>
 __device__ __forceinline__ void gemm_phase(const float* A, int lda, const float* ascale, const float* B, int M, int N, int K,
@@ -115,7 +178,7 @@ __device__ __forceinline__ void gemm_phase(const float* A, int lda, const float*
   if (2 * t64 >= (int)gridDim.x) {
     const int tn = (N + 63) / 64;
     for (int t = blockIdx.x; t < t64; t += gridDim.x)
-      tile<64, 64>(A, lda, ascale, B, K, M, N, 0, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
+      tile64(A, lda, ascale, B, K, M, N, 0, K, (t / tn) * 64, (t % tn) * 64, sm, epi);
   } else {
     const int tn = (N + 31) / 32, t32 = ((M + 31) / 32) * tn;
     for (int t = blockIdx.x; t < t32; t += gridDim.x)
@@ -125,7 +188,7 @@ __device__ __forceinline__ void gemm_phase(const float* A, int lda, const float*
 
 template <int KS>   // depthwise kernel size (0: any, loops not unrolled)
 __global__ void __launch_bounds__(MB_THREADS, 1) mbconv_kernel(const __grid_constant__ MbParams P) {
-  __shared__ float tsm[2 * 16 * 65];   // GEMM operand slabs
+  __shared__ __align__(16) float tsm[2 * 16 * 68];   // GEMM operand slabs
   __shared__ float pool[MB_MAX_E];
   __shared__ float g[MB_MAX_E];
   extern __shared__ float dyn[];       // data reuse: [pix_blk][E] depthwise output, then [cout][E + 1] Wp
