@@ -228,9 +228,9 @@ __global__ void __launch_bounds__(RX_THREADS, 1) resnext_kernel(const __grid_con
   }
   stamp(P, 1);
   grid_sync(P, 0);
-  // ---- 2: grouped 3x3 convolution (+ BN + ReLU) at the strided output pixels; (pixel, channel) pairs
-  // spread over the grid, consecutive threads = consecutive output channels
-  {
+  // ---- 2 (cg >= 8): one thread per (pixel, output channel), consecutive threads = consecutive
+  // channels; the quad mapping below measured slower here (fewer threads, 4x the weight loads each)
+  if constexpr (CG != 4) {
     const int64_t total = (int64_t)HWo * w;
     for (int64_t idx = (int64_t)blockIdx.x * RX_THREADS + tid; idx < total; idx += (int64_t)gridDim.x * RX_THREADS) {
       const int q = (int)(idx / w), o = (int)(idx % w);
@@ -254,6 +254,45 @@ __global__ void __launch_bounds__(RX_THREADS, 1) resnext_kernel(const __grid_con
         acc += part;
       }
       P.d[idx] = fmaxf(acc * __ldg(P.s2 + o) + __ldg(P.b2 + o), 0.f);
+    }
+  } else
+  // ---- 2 (cg == 4): grouped 3x3 convolution (+ BN + ReLU) at the strided output pixels: a thread
+  // computes the 4 output channels of one group (its tap reads of a -- cg channels per tap, float4 -- are
+  // shared by the 4 outputs, 4 independent accumulation chains); consecutive threads = consecutive
+  // channel quads of a pixel (coalesced float4 stores of d)
+  {
+    const int wq = w / 4;
+    const int64_t total = (int64_t)HWo * wq;
+    for (int64_t idx = (int64_t)blockIdx.x * RX_THREADS + tid; idx < total; idx += (int64_t)gridDim.x * RX_THREADS) {
+      const int q = (int)(idx / wq), o0 = 4 * (int)(idx % wq);
+      const int g = o0 / cg, oo = o0 % cg;
+      const int hs = (q / Ho) * s, ws = (q % Ho) * s;   // the pixel in the stride-1 grid
+      float acc[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+      for (int t = 0; t < RX_TAPS; ++t) {
+        const int i = t / 3, j = t % 3;
+        const int hh = (hs + i - 1 + H) % H, ww = (ws + j - 1 + H) % H;
+        const float* ar = P.a + (int64_t)(hh * H + ww) * w + g * cg;
+        const float* wr = P.W2[t] + ((int64_t)g * cg + oo) * cg;
+        float part[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll 4
+        for (int ii = 0; ii < cg; ii += 4) {
+          const float4 av = ld_ca4(ar + ii);
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const float4 wv = __ldg(reinterpret_cast<const float4*>(wr + u * cg + ii));
+            part[u] = fmaf(av.x, wv.x, fmaf(av.y, wv.y, fmaf(av.z, wv.z, fmaf(av.w, wv.w, part[u]))));
+          }
+        }
+        const float mk = P.m[t] ? __ldg(P.m[t] + hs * H + ws) : 1.f;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) acc[u] = fmaf(part[u], mk, acc[u]);
+      }
+      const float4 sc = __ldg(reinterpret_cast<const float4*>(P.s2 + o0));
+      const float4 bi = __ldg(reinterpret_cast<const float4*>(P.b2 + o0));
+      *reinterpret_cast<float4*>(P.d + (int64_t)q * w + o0) =
+          make_float4(fmaxf(acc[0] * sc.x + bi.x, 0.f), fmaxf(acc[1] * sc.y + bi.y, 0.f), fmaxf(acc[2] * sc.z + bi.z, 0.f),
+                      fmaxf(acc[3] * sc.w + bi.w, 0.f));
     }
   }
   stamp(P, 2);
