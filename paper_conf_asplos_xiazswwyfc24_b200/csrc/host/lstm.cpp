@@ -142,6 +142,14 @@ void lstm_match(const Graph& g, const Analysis& an, const souffle_device_desc& d
   const int sms = dev.num_sms > 0 ? dev.num_sms : 148;
   const int np_min = (lp.H + LSTM_UNITS - 1) / LSTM_UNITS;
   lp.NP = std::max(np_min, std::min(sms / lp.L, lp.H / 8));
+  // register-resident GEMV (K <= 512): the fewest CTAs per layer whose units fit the register layout
+  // (<= 20 units) -- fewer producers per wavefront step to wait for (10 x 256: 13 CTAs per layer,
+  // 170 vs 174 us at 14)
+  {
+    const char* fs = std::getenv("SOUFFLE_LSTM_SMEM");
+    const int np_reg = std::max(np_min, (lp.H + LSTM_REG_UNITS - 1) / LSTM_REG_UNITS);
+    if (std::max(lp.I, lp.H) + lp.H <= LSTM_REG_K && np_reg * lp.L <= sms && !(fs && std::atoi(fs))) lp.NP = np_reg;
+  }
   if (const char* e = std::getenv("SOUFFLE_LSTM_NP")) {   // timing studies
     const int v = std::atoi(e);
     if (v >= np_min && v * lp.L <= sms && v <= lp.H) lp.NP = v;
